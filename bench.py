@@ -1,0 +1,391 @@
+#!/usr/bin/env python3
+"""Benchmark: bitsliced MICKEY 2.0 keystream Tb/s on B200 (BASELINE.json).
+
+Workload (BASELINE.json configs[1]): 2^22 MICKEY 2.0 instances x 2^20 keystream
+bits per instance per GPU, keys/IVs from the seeded SplitMix64 recipe (seed
+0x5EED2020), synthetic.  One "step" = the whole hot path over one batch:
+  a-1 key/IV slicing + a-2 preclock (bsrng_rekey from device-resident keys),
+  a-3 clock loop + a-4 output + a-5 state carry (bsrng_generate).
+Headline mode "consume": CHECKSUM layout, every keystream bit is computed and
+folded into a checksum read back at the end.  Mode "materialise": ROW_MAJOR
+keystream written to HBM, 2^15 bits per call (16 GiB buffer, 32 calls/step).
+
+Multi-GPU (torchrun, one process per GPU): rank r owns global instances
+[r*n, (r+1)*n) -- weak scaling, no data-path collective; NCCL only carries the
+max step time and the uint64 checksum sum (outside the timed region).
+
+`--impl reference` times the CPU oracle (oracle/, bit-serial C) on this box's
+host cores on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+N_DEFAULT = 1 << 22
+BITS_DEFAULT = 1 << 20
+LOP3_PER_CLOCK = 327           # DESIGN.md / SURVEY App. D: algorithmic ops per clock per group
+ALU_LANES_PER_SM_CLK = 64      # 4 SMSP x 16 lanes (alu pipe rt = 2 cycles/warp-instr)
+METRIC = "MICKEY 2.0 keystream Tb/s (1 and 8 B200); fraction of LOP3/HBM roofline"
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=3)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--n", type=int, default=N_DEFAULT, help="instances per GPU")
+    p.add_argument("--bits", type=int, default=BITS_DEFAULT, help="keystream bits per instance per step")
+    p.add_argument("--mode", default="consume", choices=["consume", "materialise"],
+                   help="headline mode")
+    p.add_argument("--no-other-mode", action="store_true", help="skip timing the non-headline mode")
+    p.add_argument("--chunk-bits", type=int, default=1 << 15, help="materialise bits per call")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--sched", type=int, default=None)
+    p.add_argument("--seg-clocks", type=int, default=None)
+    p.add_argument("--ctas-per-sm", type=int, default=None)
+    return p.parse_args()
+
+
+# ------------------------------------------------------------------ helpers
+class ClockSampler:
+    """nvidia-smi clocks/throttle sampling during the timed region."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                 "-lms", "200"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except FileNotFoundError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx.append(float(f[2]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": float(np.median(sm)) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f)
+    except OSError:
+        return {}
+
+
+def profile_traffic():
+    """dram bytes per launch of the keystream kernel from the committed ncu capture."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "keystream_traffic.json")) as f:
+            return json.load(f)
+    except OSError:
+        return None
+
+
+def cpu_cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:  # pragma: no cover
+        return os.cpu_count() or 1
+
+
+def cpu_model():
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def oracle_sample(n_inst, bits, first=0, threads=None):
+    """Time the oracle (unmodified, bit-serial) on host cores; returns bits/s."""
+    import oracle
+    from paper_conf_icppw_monfaredhkzrg20_b200 import inputs
+    keys, ivs = inputs.make_inputs("mickey2", n_inst, first)
+    t = time.perf_counter()
+    oracle.mickey2_keystream_batch(keys, ivs, 80, bits, threads=threads)
+    dt = time.perf_counter() - t
+    return n_inst * bits / dt, dt
+
+
+# ------------------------------------------------------------ reference arm
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    cores = cpu_cores()
+    n_s, bits_s = 4 * cores, 1 << 14
+    for _ in range(args.warmup):
+        oracle_sample(n_s, bits_s, threads=cores)
+    tot_bits, tot_t = 0, 0.0
+    for _ in range(args.steps):
+        r, dt = oracle_sample(n_s, bits_s, threads=cores)
+        tot_bits += n_s * bits_s
+        tot_t += dt
+    v = tot_bits / tot_t / 1e12
+    line = {
+        "impl": "reference", "metric": METRIC, "value": v, "unit": "Tb/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot_t / args.steps * 1e3,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
+        "data": "synthetic (SplitMix64 keys/IVs, seed 0x5EED2020)",
+        "config": {"workload": f"configs[1]: MICKEY 2.0, {args.n} instances x {args.bits} bits per GPU "
+                               f"(reference step = bounded sample)", "mode": "bit-serial oracle"},
+        "cpu_baseline": {"value": v, "unit": "Tb/s", "cores": cores, "kind": "oracle",
+                         "sample": f"{n_s} instances x {bits_s} bits per step, {cpu_model()}"},
+        "e2e": {"value": v, "unit": "Tb/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# ----------------------------------------------------------------- our arm
+def run_ours(args, rank, world, local_rank):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_icppw_monfaredhkzrg20_b200 import bsrng, inputs
+
+    dev = torch.device("cuda", local_rank)
+    torch.cuda.set_device(dev)
+    n, bits = args.n, args.bits
+    first = rank * n
+    stream = torch.cuda.Stream(dev)
+
+    keys_h, ivs_h = inputs.make_inputs("mickey2", n, first)
+    keys_pin = torch.from_numpy(keys_h).pin_memory()
+    ivs_pin = torch.from_numpy(ivs_h).pin_memory()
+    keys_d = keys_pin.to(dev)
+    ivs_d = ivs_pin.to(dev)
+
+    with torch.cuda.stream(stream):
+        g = bsrng.Generator("mickey2", keys_d, ivs_d, first_instance=first, stream=stream)
+    for k, v in (("sched", args.sched), ("seg_clocks", args.seg_clocks), ("ctas_per_sm", args.ctas_per_sm)):
+        if v is not None:
+            g.set_option(k, v)
+    cs_out = torch.zeros(1, dtype=torch.int64, device=dev)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    def step_consume(ev=None):
+        g.rekey(keys_d, ivs_d, stream=stream)
+        if ev:
+            ev[0].record(stream)
+        g.generate(cs_out, bits, "checksum", stream=stream)
+        if ev:
+            ev[1].record(stream)
+
+    chunk = min(args.chunk_bits, bits)
+    rm_buf = None
+
+    def step_materialise(ev=None):
+        nonlocal rm_buf
+        if rm_buf is None:
+            rm_buf = torch.empty(g.out_bytes(chunk, "row_major"), dtype=torch.uint8, device=dev)
+        g.rekey(keys_d, ivs_d, stream=stream)
+        if ev:
+            ev[0].record(stream)
+        for _ in range(bits // chunk):
+            g.generate(rm_buf, chunk, "row_major", stream=stream)
+        if ev:
+            ev[1].record(stream)
+
+    def timed(step_fn, steps, warmup, sampler=None):
+        for _ in range(warmup):
+            step_fn()
+        torch.cuda.synchronize(dev)
+        step_ms, kern_ms = [], []
+        l0 = bsrng.launch_count()
+        if sampler:
+            sampler.start()
+        for _ in range(steps):
+            flush.zero_()  # L2 flush between timed steps (outside the timed region)
+            torch.cuda.synchronize(dev)
+            barrier()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            k0, k1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            step_fn((k0, k1))
+            e1.record(stream)
+            torch.cuda.synchronize(dev)
+            barrier()
+            step_ms.append(e0.elapsed_time(e1))
+            kern_ms.append(k0.elapsed_time(k1))
+        clocks = sampler.stop() if sampler else None
+        launches = bsrng.launch_count() - l0
+        t = torch.tensor([sum(step_ms), sum(kern_ms)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t[0]) / steps, float(t[1]) / steps, launches, clocks
+
+    peaks = measured_peaks()
+    sm_max = float(peaks.get("sm_max_mhz", 1965.0))
+    nsm = torch.cuda.get_device_properties(dev).multi_processor_count
+
+    def roofline(kern_ms_per_step, clocks):
+        lop3 = LOP3_PER_CLOCK * (n // 32) * bits       # algorithmic LOP3 per step, dominant kernel(s)
+        achieved = lop3 / (kern_ms_per_step * 1e-3) / 1e12
+        peak = nsm * ALU_LANES_PER_SM_CLK * sm_max * 1e6 / 1e12
+        out = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TLOP3/s", "frac": achieved / peak,
+               "peak_basis": f"{nsm} SMs x {ALU_LANES_PER_SM_CLK} LOP3 lanes/clk x sm_max {sm_max:.0f} MHz "
+                             "(B300_MICROARCH alu pipe rt=2/SMSP; DESIGN.md)",
+               "traffic": None}
+        if clocks and clocks.get("sm_mhz"):
+            out["frac_at_sampled_clock"] = achieved / (nsm * ALU_LANES_PER_SM_CLK * clocks["sm_mhz"] * 1e6 / 1e12)
+        return out
+
+    results = {}
+    modes = [args.mode] + ([] if args.no_other_mode else [m for m in ("consume", "materialise") if m != args.mode])
+    for mode in modes:
+        fn = step_consume if mode == "consume" else step_materialise
+        sampler = ClockSampler(local_rank) if (rank == 0 and mode == args.mode) else None
+        ms, kms, launches, clocks = timed(fn, args.steps, args.warmup, sampler)
+        tbps = world * n * bits / (ms * 1e-3) / 1e12
+        res = {"value": tbps, "ms_per_step": ms, "kernel_ms_per_step": kms,
+               "kernel_tbps_per_gpu": n * bits / (kms * 1e-3) / 1e12,
+               "gpu_launches": launches, "roofline": roofline(kms, clocks)}
+        if mode == "materialise":
+            out_bytes = n * bits / 8
+            res["hbm_write_gbs_per_gpu"] = out_bytes / (kms * 1e-3) / 1e9
+            res["hbm_write_frac"] = res["hbm_write_gbs_per_gpu"] / float(peaks.get("hbm_gbs", 6650.0))
+            res["calls_per_step"] = bits // chunk
+        if clocks:
+            res["clocks"] = clocks
+        results[mode] = res
+
+    # checksum of one consume step (sharding invariant), outside the timed region
+    step_consume()
+    torch.cuda.synchronize(dev)
+    cs = cs_out.clone()
+    if world > 1:
+        dist.all_reduce(cs, op=dist.ReduceOp.SUM)
+    checksum = int(cs.item()) & ((1 << 64) - 1)
+
+    # e2e: host keys (pinned) -> rekey through the C ABI -> CHECKSUM -> 8 B back to host
+    e2e = None
+    if not args.no_e2e:
+        cs_host = torch.zeros(1, dtype=torch.int64).pin_memory()
+
+        def step_e2e(ev=None):
+            g.rekey(keys_pin.numpy(), ivs_pin.numpy(), stream=stream)
+            if ev:
+                ev[0].record(stream)
+            g.generate(cs_out, bits, "checksum", stream=stream)
+            if ev:
+                ev[1].record(stream)
+            with torch.cuda.stream(stream):
+                cs_host.copy_(cs_out, non_blocking=True)
+
+        ms_e2e, _, _, _ = timed(step_e2e, max(1, args.steps), 1)
+        e2e = {"value": world * n * bits / (ms_e2e * 1e-3) / 1e12, "unit": "Tb/s",
+               "h2d_bytes_per_step": int(keys_h.nbytes + ivs_h.nbytes), "d2h_bytes_per_step": 8,
+               "ms_per_step": ms_e2e, "mode": "consume"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cores = cpu_cores()
+        n_s, bits_s = 8 * cores, 1 << 16
+        r, dt = oracle_sample(n_s, bits_s, threads=cores)
+        cpu = {"value": r / 1e12, "unit": "Tb/s", "cores": cores, "kind": "oracle",
+               "sample": f"{n_s} instances x {bits_s} bits ({dt:.1f} s), first instances of the workload, "
+                         f"{cpu_model()}", "bits_per_s_per_core": r / cores}
+
+    if rank == 0:
+        head = results[args.mode]
+        rf = head["roofline"]
+        tr = profile_traffic()
+        if tr and tr.get("mode") == args.mode and tr.get("n") == n:
+            rf["traffic"] = tr.get("dram_bytes_per_launch")
+            rf["traffic_note"] = tr.get("note")
+        line = {
+            "metric": METRIC, "value": head["value"], "unit": "Tb/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": head["ms_per_step"],
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
+            "data": "synthetic (SplitMix64 keys/IVs, seed 0x5EED2020)",
+            "config": {"workload": f"configs[1]: MICKEY 2.0, {n} instances x {bits} bits per GPU per step "
+                                   f"({args.mode})", "instances_per_gpu": n, "bits_per_instance": bits,
+                       "mode": args.mode, "parallelism": f"instance-range shards x{world}",
+                       "l2": "flushed (256 MiB write) between timed steps; state 100 MiB, keys 80 MiB"},
+            "roofline": rf, "clocks": head.get("clocks"), "gpu_launches": head["gpu_launches"],
+            "e2e": e2e, "cpu_baseline": cpu, "checksum": f"{checksum:016x}",
+            "modes": {m: {k: v for k, v in r.items() if k != "clocks"} for m, r in results.items()},
+            "paper_context": "2.72 Tb/s RTX 2080 Ti, 2.90 Tb/s V100 (PAPER.md:46-50, 852-854); "
+                             "exceeds the bit-exact LOP3 bound on those GPUs, see BASELINE.md",
+        }
+        print(json.dumps(line), flush=True)
+    g.close()
+
+
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus and world == 1 and args.gpus > 1:
+        print(f"--gpus {args.gpus} needs torchrun (WORLD_SIZE={world})", file=sys.stderr)
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    try:
+        run_ours(args, rank, world, local_rank)
+    finally:
+        if world > 1:
+            import torch.distributed as dist
+            dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

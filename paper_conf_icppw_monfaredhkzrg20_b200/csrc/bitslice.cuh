@@ -1,0 +1,102 @@
+// bitslice.cuh -- layout conversions for the column-major ("bitsliced")
+// representation, sm_100a.
+//
+// PAPER.md:478-489 (sec. 4.1): "a batch of 32 bits data stored in a single
+// register, represents state bits from 32 uncorrelated different parallel
+// LFSRs having the same bit significance".  Lane j of a slice word is instance
+// 32g + j of group g (reading R8).
+#pragma once
+#include <cstdint>
+
+namespace bsk {
+
+// ---------------------------------------------------------------------------
+// Key/IV slicing (SURVEY step a-1; "32x80 bits of IV for each
+// thread").  One warp per group g: lane j holds instance 32g+j's byte string;
+// one __ballot_sync per bit position gathers the 32 lanes into a slice word.
+//   raw   : uint8 [n][NBYTES] row-major (device)
+//   out   : uint32 [NBITS][Gp]  (bit b of instance 32g+j -> bit j of out[b][g])
+//   MSB   : bit b of a byte string is (byte[b/8] >> (7 - b%8)) & 1 if true
+//           (MICKEY, spec [5]), (byte[b/8] >> (b%8)) & 1 otherwise (Grain)
+// Instances >= n (padding) get all-zero bytes.
+// ---------------------------------------------------------------------------
+template <int NBYTES, int NBITS, bool MSB>
+__global__ void __launch_bounds__(256) slice_bits_kernel(const uint8_t* __restrict__ raw,
+                                                         uint64_t n, uint32_t* __restrict__ out,
+                                                         uint64_t Gp)
+{
+    const uint64_t warp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t lane = threadIdx.x & 31u;
+    if (warp >= Gp) return;  // warp-uniform
+    const uint64_t inst = warp * 32u + lane;
+    uint8_t b[NBYTES];
+#pragma unroll
+    for (int i = 0; i < NBYTES; ++i) b[i] = (inst < n) ? raw[inst * NBYTES + i] : uint8_t(0);
+#pragma unroll
+    for (int bit = 0; bit < NBITS; ++bit) {
+        const uint32_t v = MSB ? (b[bit >> 3] >> (7 - (bit & 7))) & 1u : (b[bit >> 3] >> (bit & 7)) & 1u;
+        const uint32_t w = __ballot_sync(0xffffffffu, v);
+        if (lane == uint32_t(bit & 31)) out[uint64_t(bit) * Gp + warp] = w;
+    }
+}
+
+// ---------------------------------------------------------------------------
+// 32x32 bit transpose, one thread, in registers (SURVEY step a-4 (iii)).
+// Input rows x[q] (q = 0..N-1) are a slab of the 32x32 matrix A after the
+// stage-16 PRMT split; output x[q] = B[.] with B[c] bit r = A[r] bit c.
+// Stages s = 8 (PRMT byte shuffle), 4, 2, 1 (shift + LOP3 select) on row pairs
+// (r, r+s), r & s == 0.  16 rows -> 8 + 3*16 = 56... ops, all ALU.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ void bt_stage8(uint32_t& a, uint32_t& b)
+{
+    const uint32_t na = __byte_perm(a, b, 0x6240);
+    const uint32_t nb = __byte_perm(a, b, 0x7351);
+    a = na;
+    b = nb;
+}
+
+template <int S, uint32_t M>
+__device__ __forceinline__ void bt_stage(uint32_t& a, uint32_t& b)
+{
+    // element (r, c | S) <-> (r + S, c), c & S == 0; M = bits with c & S == 0
+    const uint32_t na = (a & M) | ((b << S) & ~M);
+    const uint32_t nb = ((a >> S) & M) | (b & ~M);
+    a = na;
+    b = nb;
+}
+
+// Transpose the 16-row half produced by the stage-16 split.
+__device__ __forceinline__ void bt_transpose16(uint32_t (&x)[16])
+{
+#pragma unroll
+    for (int r = 0; r < 16; ++r)
+        if ((r & 8) == 0) bt_stage8(x[r], x[r + 8]);
+#pragma unroll
+    for (int r = 0; r < 16; ++r)
+        if ((r & 4) == 0) bt_stage<4, 0x0F0F0F0Fu>(x[r], x[r + 4]);
+#pragma unroll
+    for (int r = 0; r < 16; ++r)
+        if ((r & 2) == 0) bt_stage<2, 0x33333333u>(x[r], x[r + 2]);
+#pragma unroll
+    for (int r = 0; r < 16; ++r)
+        if ((r & 1) == 0) bt_stage<1, 0x55555555u>(x[r], x[r + 1]);
+}
+
+// Hide a pointer's provenance from the optimiser (no code emitted beyond a
+// register move), so address arithmetic is not hoisted/CSE'd across the
+// register-resident clock loop.
+template <class T>
+__device__ __forceinline__ T* opaque(T* p)
+{
+    asm volatile("" : "+l"(p));
+    return p;
+}
+
+__device__ __forceinline__ uint64_t fmix64(uint64_t z)
+{
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+}  // namespace bsk

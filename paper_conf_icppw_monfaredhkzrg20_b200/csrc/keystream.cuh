@@ -1,0 +1,241 @@
+// keystream.cuh -- the register-resident keystream clock loop (SURVEY steps a-3,
+// a-4, a-5), generic over a bitsliced cipher C, for sm_100a.
+//
+// One thread = one group of 32 instances = one slice word per state bit
+// (PAPER.md:618-626).  The whole state lives in registers across all clocks of
+// a work item ("do not require any additional memory rather
+// than registers"); it touches HBM only at item entry/exit (state carry, a-5).
+//
+// Work distribution (B200 design, not the paper's): a persistent grid sized to
+// the resident-warp capacity of the 148 SMs pulls work items from an atomic
+// ticket.  Item k = (segment k / units, warp-unit k % units): 32 groups for
+// seg_clocks clocks.  Segment s of a unit waits for segment s-1 of the same
+// unit (flag), so a call is split in time as well as across instances and the
+// last wave's tail is one segment long instead of one whole call.  Tickets are
+// taken in order by resident warps, so every awaited item is held by a running
+// warp: no deadlock.
+//
+// Output layouts (sec. 4.5: registers -> shared memory ->
+// coalesced global stores):
+//   CHECKSUM : acc ^= z (fused into the output LOP3); fmix64 + warp sum + one
+//              atomicAdd per warp at the end of the call.
+//   SLICED   : out[t][g] = z -- one coalesced STG.32 per clock (128 B per warp).
+//   ROW_MAJOR: z -> shared memory (one conflict-free STS per clock); every 32
+//              clocks each thread reloads its 32 words, transposes the 32x32
+//              bit block in registers (PRMT + shift/LOP3 butterfly, split in
+//              two 16-row halves to bound register pressure) and writes one
+//              32-bit word per instance row.
+#pragma once
+#include <cstdint>
+
+#include "bitslice.cuh"
+
+namespace bsk {
+
+enum : int { L_ROW_MAJOR = 0, L_SLICED = 1, L_CHECKSUM = 2 };
+
+struct KsArgs {
+    uint32_t* state;      // [C::NSTATE + 1][Gp] (last row: checksum accumulator)
+    uint64_t Gp;          // padded groups (multiple of 32) = 32 * units
+    uint64_t G;           // real groups
+    uint64_t n;           // real instances
+    uint32_t tail_mask;   // valid lanes of group G-1
+    uint64_t nclocks;     // clocks in this call (multiple of 32)
+    uint64_t t0;          // clocks generated before this call
+    uint64_t g_base;      // global index of group 0 (checksum)
+    void* out;
+    uint64_t row_bytes;   // ROW_MAJOR row stride = nclocks / 8
+    uint64_t seg_clocks;  // clocks per work item (multiple of 32)
+    uint64_t nseg;        // segments per call
+    uint64_t units;       // warp-units = Gp / 32
+    uint32_t* ticket;     // persistent mode: [1], zeroed before launch
+    uint32_t* flags;      // persistent mode: [units], zeroed before launch
+    unsigned long long* dbg;  // optional scheduler counters (BSRNG_DEBUG), or null
+    int persistent;
+};
+
+__device__ __forceinline__ uint32_t ld_acquire(const uint32_t* p)
+{
+    uint32_t v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release(uint32_t* p, uint32_t v)
+{
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+__device__ __forceinline__ uint32_t lane_mask(const KsArgs& a, uint64_t g)
+{
+    return g + 1 < a.G ? 0xFFFFFFFFu : (g + 1 == a.G ? a.tail_mask : 0u);
+}
+
+// Transpose the 32 staged slice words zs[t][lane] (t = 0..31) of this thread
+// and store its instance rows.  Row t of the bit matrix is clock t, or clock
+// t^7 for MSB-first ciphers so that clock 8b+q lands in bit 7-q of byte b.
+//   row0  : address of (instance 32g, this 32-clock block) in the output
+//   nvalid: rows of this group that are real instances (0..32)
+template <bool MSB_FIRST>
+__device__ __forceinline__ void rowmajor_flush(const uint32_t* zs, uint8_t* row0, uint64_t row_bytes,
+                                               uint32_t nvalid)
+{
+    constexpr int X = MSB_FIRST ? 7 : 0;
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+        uint32_t x[16];
+#pragma unroll
+        for (int q = 0; q < 16; ++q) {
+            const uint32_t lo = zs[((q ^ X)) * 32];
+            const uint32_t hi = zs[((q + 16) ^ X) * 32];
+            x[q] = __byte_perm(lo, hi, h == 0 ? 0x5410 : 0x7632);
+        }
+        bt_transpose16(x);
+#pragma unroll
+        for (int q = 0; q < 16; ++q)
+            if (uint32_t(16 * h + q) < nvalid)
+                *reinterpret_cast<uint32_t*>(row0 + uint64_t(16 * h + q) * row_bytes) = x[q];
+    }
+}
+
+__device__ __forceinline__ uint32_t laneid_volatile()
+{
+    uint32_t v;
+    asm volatile("mov.u32 %0, %%laneid;" : "=r"(v));
+    return v;
+}
+
+// Fetch the next work item for this warp into smem (persistent mode).
+__device__ __forceinline__ void next_item(const KsArgs& a, volatile uint32_t* slot)
+{
+    __syncwarp();
+    if (laneid_volatile() == 0) *slot = atomicAdd(a.ticket, 1u);
+    __syncwarp();
+}
+
+template <class C, int LAYOUT, int U, int BLOCK>
+__global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
+{
+    static_assert(32 % U == 0, "U must divide 32");
+    constexpr int NW = BLOCK / 32;
+    __shared__ uint32_t zs_all[LAYOUT == L_ROW_MAJOR ? NW * 32 * 32 : 1];
+    __shared__ uint32_t s_item[NW];
+    // Only `s_item` (smem) and the loop counters survive a clock loop; every
+    // other per-item value is re-derived afterwards, so the 200 state words
+    // plus temporaries fit in 255 registers without spilling.
+    volatile uint32_t* slot = s_item + (threadIdx.x >> 5);
+    if (a.persistent)
+        next_item(a, slot);
+    else if (laneid_volatile() == 0)
+        *slot = (blockIdx.x * BLOCK + threadIdx.x) >> 5;
+    __syncwarp();
+
+    const uint64_t total = a.units * a.nseg;
+    for (;;) {
+        uint64_t item = *slot;
+        if (item >= total) break;
+        uint32_t lane = laneid_volatile();
+        uint64_t seg = item / a.units;
+        uint64_t w = item - seg * a.units;
+        uint64_t g = w * 32u + lane;
+        if (seg > 0) {
+            if (lane == 0)
+            {
+                uint32_t spins = 0;
+                while (ld_acquire(a.flags + w) < seg) {
+                    __nanosleep(256);
+                    ++spins;
+                }
+                if (a.dbg) {
+                    atomicAdd(a.dbg + 0, 1ull);
+                    if (spins) atomicAdd(a.dbg + 1, 1ull);
+                    atomicAdd(a.dbg + 2, (unsigned long long)spins);
+                }
+            }
+            __syncwarp();
+            (void)ld_acquire(a.flags + w);
+        }
+        const uint64_t clk_begin = seg * a.seg_clocks;
+        const uint64_t left = a.nclocks - clk_begin;
+        const uint32_t nclk = uint32_t(left < a.seg_clocks ? left : a.seg_clocks);
+
+        C c;
+        c.load(a.state, a.Gp, g);
+        uint32_t acc = 0;
+        if (LAYOUT == L_CHECKSUM && seg > 0) acc = __ldcg(a.state + uint64_t(C::NSTATE) * a.Gp + g);
+
+        if (LAYOUT == L_CHECKSUM) {
+#pragma unroll 1
+            for (uint32_t it = nclk / U; it != 0; --it) {
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    acc ^= c.z();
+                    c.clock();
+                }
+            }
+        } else if (LAYOUT == L_SLICED) {
+            const uint32_t m = lane_mask(a, g);
+            uint32_t* o = static_cast<uint32_t*>(a.out) + clk_begin * a.G + (g < a.G ? g : 0);
+            const uint64_t stride = g < a.G ? a.G : 0;  // 0 = padding group: never stores
+#pragma unroll 1
+            for (uint32_t it = nclk / U; it != 0; --it) {
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    const uint32_t z = c.z() & m;
+                    if (stride) __stcs(o, z);
+                    o += stride;
+                    c.clock();
+                }
+            }
+        } else {  // ROW_MAJOR
+            const uint64_t first = g * 32u;
+            const uint32_t nvalid = first >= a.n ? 0u : uint32_t(a.n - first < 32 ? a.n - first : 32);
+            uint8_t* row0 = static_cast<uint8_t*>(a.out) + (nvalid ? first : 0) * a.row_bytes + (clk_begin >> 3);
+            uint32_t* zs = zs_all + (threadIdx.x >> 5) * 32 * 32 + lane;
+#pragma unroll 1
+            for (uint32_t blk = nclk / 32; blk != 0; --blk) {
+#pragma unroll 1
+                for (uint32_t k = 0; k < 32; k += U) {
+#pragma unroll
+                    for (int u = 0; u < U; ++u) {
+                        zs[(k + u) * 32] = c.z();
+                        c.clock();
+                    }
+                }
+                rowmajor_flush<C::MSB_FIRST>(zs, row0, a.row_bytes, nvalid);
+                row0 += 4;
+            }
+        }
+
+        // re-derive the item context (kept out of registers during the loop)
+        item = *slot;
+        lane = laneid_volatile();
+        seg = item / a.units;
+        w = item - seg * a.units;
+        g = w * 32u + lane;
+        const bool last = (seg + 1 == a.nseg);
+        if (LAYOUT == L_CHECKSUM) {
+            if (last) {
+                uint64_t v = 0;
+                if (g < a.G)
+                    v = fmix64(uint64_t(acc & lane_mask(a, g)) ^ ((a.g_base + g) * 0x9E3779B97F4A7C15ull) ^
+                               (a.t0 * 0xBF58476D1CE4E5B9ull));
+#pragma unroll
+                for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(0xFFFFFFFFu, v, off);
+                if (lane == 0) atomicAdd(static_cast<unsigned long long*>(a.out), (unsigned long long)v);
+            } else {
+                __stcg(a.state + uint64_t(C::NSTATE) * a.Gp + g, acc);
+            }
+        }
+        c.store(a.state, a.Gp, g);
+
+        if (!a.persistent) break;
+        if (!last) {
+            __threadfence();
+            __syncwarp();
+            if (lane == 0) st_release(a.flags + w, uint32_t(seg + 1));
+        }
+        next_item(a, slot);
+    }
+}
+
+}  // namespace bsk

@@ -1,0 +1,163 @@
+// mickey2.cuh -- bitsliced MICKEY 2.0 for sm_100a.
+//
+// PAPER.md:597-656 (sec. 4.4, Fig. 9): "instead of two 100-bit registers ...
+// 200 registers, each containing 32 bits are employed ... each GPU thread can
+// execute 32 parallel Mickey 2.0 ciphers, and each thread at each clock cycle
+// generates 32 random bits."  The per-bit procedures are those of the MICKEY
+// 2.0 specification (ref [5]); here every bit r_i / s_i is a
+// 32-lane slice word and every step is one 3-input logic op (LOP3).
+//
+// The tables below are the GPU-side encoding (packed masks, bit i at word
+// i/32, bit i%32).  They are NOT shared with the oracle, which transcribes the
+// specification's bit rows; tests/test_oracle_mickey2.py checks the two
+// encodings agree.
+//
+// Op count per keystream clock: R 149, S 174, fb0/fb1 2,
+// control 1, output 1 = 327 LOP3 for 32 keystream bits.
+#pragma once
+#include <cstdint>
+
+#include "bitslice.cuh"
+
+namespace bsk {
+namespace m2 {
+
+__host__ __device__ constexpr uint32_t pick(uint32_t w0, uint32_t w1, uint32_t w2, uint32_t w3, int i)
+{
+    return ((i < 32 ? w0 : i < 64 ? w1 : i < 96 ? w2 : w3) >> (i & 31)) & 1u;
+}
+// RTAPS (50 taps), COMP0/COMP1 (used for 1 <= i <= 98), FB0, FB1.
+__host__ __device__ constexpr bool rtap(int i) { return pick(0x1279327Bu, 0xB5546660u, 0xDF87818Fu, 0x00000003u, i); }
+__host__ __device__ constexpr uint32_t comp0(int i) { return pick(0x6AA97A30u, 0x7942A809u, 0x057EBFEAu, 0x00000006u, i) ? 0xFFFFFFFFu : 0u; }
+__host__ __device__ constexpr uint32_t comp1(int i) { return pick(0xDD629E9Au, 0xE3A21D63u, 0x91C23DD7u, 0x00000001u, i) ? 0xFFFFFFFFu : 0u; }
+__host__ __device__ constexpr bool fb0(int i) { return pick(0x9FFA7FAFu, 0xAF4A9381u, 0x9CEC5802u, 0x00000001u, i); }
+__host__ __device__ constexpr bool fb1(int i) { return pick(0x4C8CB877u, 0x4911B063u, 0x40FBC52Bu, 0x00000008u, i); }
+
+constexpr int NSTATE = 200;
+
+// a ^ (b & c) as one explicit LOP3.  Written as inline PTX because, given the
+// C expression, the compiler folds CONTROL_BIT_R = s34 ^ r67 into every AND
+// (r_i & (s34 ^ r67) is one 3-input LOP3) and then needs a second LOP3 for the
+// XOR with r_{i-1}: 2 ops per bit instead of 1 (+50 ops per clock).
+constexpr uint32_t LUT_A_XOR_BC = 0xF0u ^ (0xCCu & 0xAAu);  // 0x78
+template <uint32_t LUT>
+__device__ __forceinline__ uint32_t lop3(uint32_t a, uint32_t b, uint32_t c)
+{
+    uint32_t d;
+    asm("lop3.b32 %0, %1, %2, %3, %4;" : "=r"(d) : "r"(a), "r"(b), "r"(c), "n"(LUT));
+    return d;
+}  // slice words of state per group: r_0..r_99, s_0..s_99
+
+// One CLOCK_KG on 32 lanes.  MIX = the spec's MIXING flag (init clocks);
+// `in` = INPUT_BIT slice word (ignored unless MIX).
+//   CONTROL_BIT_R = s34 ^ r67, CONTROL_BIT_S = s67 ^ r33   (Fig. 2)
+//   FEEDBACK_R = r99 ^ in ^ (MIX ? s50 : 0), FEEDBACK_S = s99 ^ in
+//   r'_i = r_{i-1} ^ [i in RTAPS] fbR ^ (ctlR & r_i)          (r_{-1} = 0)
+//   s'_i = s^_i ^ (FB0_i & fbS & ~ctlS) ^ (FB1_i & fbS & ctlS)
+//   s^_i = s_{i-1} ^ ((s_i ^ COMP0_i) & (s_{i+1} ^ COMP1_i)), s^_0 = 0, s^_99 = s_98
+// R is updated in place top-down (old r_i is read only by r'_i and r'_{i+1});
+// S goes through a renamed array (every old s_i is read by three updates), which
+// after full unrolling is pure register renaming.
+template <bool MIX>
+__device__ __forceinline__ void clock_kg(uint32_t (&r)[100], uint32_t (&s)[100], uint32_t in)
+{
+    const uint32_t ctl_r = s[34] ^ r[67];
+    const uint32_t ctl_s = s[67] ^ r[33];
+    const uint32_t fb_r = MIX ? (r[99] ^ in ^ s[50]) : r[99];
+    const uint32_t fb_s = MIX ? (s[99] ^ in) : s[99];
+    const uint32_t fb_s0 = fb_s & ~ctl_s;  // FB0 taps apply where CONTROL_BIT_S = 0
+    const uint32_t fb_s1 = fb_s & ctl_s;   // FB1 taps apply where CONTROL_BIT_S = 1
+
+#pragma unroll
+    for (int i = 99; i >= 1; --i) {
+        const uint32_t a = rtap(i) ? (r[i - 1] ^ fb_r) : r[i - 1];
+        r[i] = lop3<LUT_A_XOR_BC>(a, ctl_r, r[i]);
+    }
+    r[0] = lop3<LUT_A_XOR_BC>(fb_r, ctl_r, r[0]);  // 0 is in RTAPS
+
+    uint32_t ns[100];
+#pragma unroll
+    for (int i = 0; i < 100; ++i) {
+        uint32_t v;
+        if (i == 0)
+            v = 0u;
+        else if (i == 99)
+            v = s[98];
+        else
+            v = s[i - 1] ^ ((s[i] ^ comp0(i)) & (s[i + 1] ^ comp1(i)));
+        if (fb0(i) && fb1(i))
+            v ^= fb_s;
+        else if (fb0(i))
+            v ^= fb_s0;
+        else if (fb1(i))
+            v ^= fb_s1;
+        ns[i] = v;
+    }
+#pragma unroll
+    for (int i = 0; i < 100; ++i) s[i] = ns[i];
+}
+
+}  // namespace m2
+}  // namespace bsk
+
+namespace bsk {
+
+// Cipher traits used by keystream_kernel (keystream.cuh).
+struct Mickey2 {
+    static constexpr int NSTATE = m2::NSTATE;
+    static constexpr bool MSB_FIRST = true;  // spec [5]: keystream packed MSB-first
+    uint32_t r[100], s[100];
+
+    // State carry (SURVEY step a-5).  The row pointer goes through opaque()
+    // so the 200 load addresses are not kept live across the clock loop for
+    // reuse by the stores (that would cost 400 registers).
+    __device__ __forceinline__ void load(const uint32_t* st, uint64_t Gp, uint64_t g)
+    {
+        const uint32_t* p = opaque(st + g);
+#pragma unroll
+        for (int i = 0; i < 100; ++i) r[i] = __ldcg(p + uint64_t(i) * Gp);
+#pragma unroll
+        for (int i = 0; i < 100; ++i) s[i] = __ldcg(p + uint64_t(100 + i) * Gp);
+    }
+    __device__ __forceinline__ void store(uint32_t* st, uint64_t Gp, uint64_t g) const
+    {
+        uint32_t* p = opaque(st + g);
+#pragma unroll
+        for (int i = 0; i < 100; ++i) __stcg(p + uint64_t(i) * Gp, r[i]);
+#pragma unroll
+        for (int i = 0; i < 100; ++i) __stcg(p + uint64_t(100 + i) * Gp, s[i]);
+    }
+    // keystream bit z = r0 ^ s0, taken before the clock (spec [5])
+    __device__ __forceinline__ uint32_t z() const { return r[0] ^ s[0]; }
+    __device__ __forceinline__ void clock() { m2::clock_kg<false>(r, s, 0u); }
+};
+
+// Initialisation (SURVEY step a-2, spec [5]): R = S = 0,
+// then CLOCK_KG(MIXING=1, INPUT_BIT) for the iv_bits IV bits, the 80 key bits
+// and 100 zero bits.  One thread per group; one coalesced slice word per clock.
+//   iv_s, key_s: uint32 [80][Gp] sliced bits (slice_bits_kernel)
+//   state      : uint32 [201][Gp] (row 200 = checksum accumulator, zeroed)
+__global__ void __launch_bounds__(128) m2_preclock_kernel(const uint32_t* __restrict__ iv_s,
+                                                          const uint32_t* __restrict__ key_s,
+                                                          int iv_bits, uint32_t* __restrict__ state,
+                                                          uint64_t Gp)
+{
+    const uint64_t g = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (g >= Gp) return;
+    uint32_t r[100], s[100];
+#pragma unroll
+    for (int i = 0; i < 100; ++i) r[i] = s[i] = 0u;
+#pragma unroll 1
+    for (int i = 0; i < iv_bits; ++i) m2::clock_kg<true>(r, s, iv_s[uint64_t(i) * Gp + g]);
+#pragma unroll 1
+    for (int i = 0; i < 80; ++i) m2::clock_kg<true>(r, s, key_s[uint64_t(i) * Gp + g]);
+#pragma unroll 1
+    for (int i = 0; i < 100; ++i) m2::clock_kg<true>(r, s, 0u);
+#pragma unroll
+    for (int i = 0; i < 100; ++i) state[uint64_t(i) * Gp + g] = r[i];
+#pragma unroll
+    for (int i = 0; i < 100; ++i) state[uint64_t(100 + i) * Gp + g] = s[i];
+    state[uint64_t(200) * Gp + g] = 0u;
+}
+
+}  // namespace bsk
