@@ -45,8 +45,12 @@ def parse():
     p.add_argument("--steps", type=int, default=3)
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    p.add_argument("--n", type=int, default=N_DEFAULT, help="instances per GPU")
-    p.add_argument("--bits", type=int, default=BITS_DEFAULT, help="keystream bits per instance per step")
+    p.add_argument("--workload", default="c2", choices=["c2", "c3"],
+                   help="c2 = BASELINE configs[1] per GPU (weak scaling); "
+                        "c3 = configs[2]: 2^25 instances x 2^18 bits = 1 TiB total, split across GPUs (strong)")
+    p.add_argument("--n", type=int, default=None, help="instances per GPU (c2) / in total (c3)")
+    p.add_argument("--bits", type=int, default=None, help="keystream bits per instance per step")
+    p.add_argument("--no-context", action="store_true", help="skip the ALU-peak / cuRAND microbenchmarks")
     p.add_argument("--mode", default="consume", choices=["consume", "materialise"],
                    help="headline mode")
     p.add_argument("--no-other-mode", action="store_true", help="skip timing the non-headline mode")
@@ -157,12 +161,59 @@ def oracle_sample(n_inst, bits, first=0, threads=None):
     return n_inst * bits / dt, dt
 
 
+def cpu_baseline(target_s=12.0):
+    """The oracle as it stands, on all host cores, on a bounded sample of the
+    workload (its first instances, 2^16 bits each) sized for ~target_s."""
+    cores = cpu_cores()
+    r0, _ = oracle_sample(2 * cores, 1 << 13, threads=cores)      # calibration
+    n_s = int(max(cores, min(1 << 16, r0 * target_s / (1 << 16))))
+    n_s = (n_s + cores - 1) // cores * cores
+    r, dt = oracle_sample(n_s, 1 << 16, threads=cores)
+    return {"value": r / 1e12, "unit": "Tb/s", "cores": cores, "kind": "oracle",
+            "sample": f"instances 0..{n_s - 1} of the workload x 65536 bits ({dt:.1f} s), {cpu_model()}",
+            "bits_per_s_per_core": r / cores}
+
+
+def run_context(local_rank):
+    """Live context numbers on this GPU: the measured LOP3 issue ceiling and
+    cuRAND on the same B200 (tools/microbench, built by __graft_entry__.build)."""
+    out = {}
+    mb = os.path.join(ROOT, "tools", "microbench")
+    env = dict(os.environ, CUDA_VISIBLE_DEVICES=os.environ.get("CUDA_VISIBLE_DEVICES", str(local_rank)))
+    for name, argv in (("alu_peak", ["200000"]), ("curand", ["4294967296"])):
+        exe = os.path.join(mb, "alu_peak" if name == "alu_peak" else "curand_bench")
+        if not os.path.exists(exe):
+            out[name] = "not built"
+            continue
+        try:
+            r = subprocess.run([exe, *argv], capture_output=True, text=True, timeout=120, env=env)
+            out[name] = [json.loads(ln) for ln in r.stdout.splitlines() if ln.startswith("{")]
+        except Exception as e:  # pragma: no cover
+            out[name] = f"failed: {e}"
+    if isinstance(out.get("alu_peak"), list) and out["alu_peak"]:
+        out["alu_peak_tlop3_per_s"] = max(x["tlop3_per_s"] for x in out["alu_peak"] if x["variant"] == "lop3")
+    return out
+
+
 # ------------------------------------------------------------ reference arm
+def workload(args, world):
+    """(n_total, bits, scaling, description) of the benchmarked configuration."""
+    if args.workload == "c2":
+        bits = args.bits or BITS_DEFAULT
+        n = args.n or N_DEFAULT
+        return n * world, bits, "weak", f"configs[1]: MICKEY 2.0, {n} instances x {bits} bits per GPU per step"
+    bits = args.bits or (1 << 18)
+    n_total = args.n or (1 << 25)
+    return n_total, bits, "strong", (f"configs[2]: MICKEY 2.0, {n_total} instances x {bits} bits in total, "
+                                     f"split over {world} GPU(s)")
+
+
 def run_reference(args, rank, world):
     if rank != 0:
         return
+    _, _, scaling, desc = workload(args, world)
     cores = cpu_cores()
-    n_s, bits_s = 4 * cores, 1 << 14
+    n_s, bits_s = 16 * cores, 1 << 15
     for _ in range(args.warmup):
         oracle_sample(n_s, bits_s, threads=cores)
     tot_bits, tot_t = 0, 0.0
@@ -174,10 +225,10 @@ def run_reference(args, rank, world):
     line = {
         "impl": "reference", "metric": METRIC, "value": v, "unit": "Tb/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot_t / args.steps * 1e3,
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
+        "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "u32",
         "data": "synthetic (SplitMix64 keys/IVs, seed 0x5EED2020)",
-        "config": {"workload": f"configs[1]: MICKEY 2.0, {args.n} instances x {args.bits} bits per GPU "
-                               f"(reference step = bounded sample)", "mode": "bit-serial oracle"},
+        "config": {"workload": f"{desc} ({args.mode})", "mode": args.mode,
+                   "reference_step": f"bounded sample: first {n_s} instances x {bits_s} bits, bit-serial oracle"},
         "cpu_baseline": {"value": v, "unit": "Tb/s", "cores": cores, "kind": "oracle",
                          "sample": f"{n_s} instances x {bits_s} bits per step, {cpu_model()}"},
         "e2e": {"value": v, "unit": "Tb/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -191,10 +242,15 @@ def run_ours(args, rank, world, local_rank):
     import torch.distributed as dist
     from paper_conf_icppw_monfaredhkzrg20_b200 import bsrng, inputs
 
+    from paper_conf_icppw_monfaredhkzrg20_b200 import shard
+
     dev = torch.device("cuda", local_rank)
     torch.cuda.set_device(dev)
-    n, bits = args.n, args.bits
-    first = rank * n
+    n_total, bits, scaling, desc = workload(args, world)
+    if args.workload == "c2":
+        first, n = shard.weak_range(rank, n_total // world)
+    else:
+        first, n = shard.strong_range(rank, world, n_total)
     stream = torch.cuda.Stream(dev)
 
     keys_h, ivs_h = inputs.make_inputs("mickey2", n, first)
@@ -288,7 +344,7 @@ def run_ours(args, rank, world, local_rank):
         fn = step_consume if mode == "consume" else step_materialise
         sampler = ClockSampler(local_rank) if (rank == 0 and mode == args.mode) else None
         ms, kms, launches, clocks = timed(fn, args.steps, args.warmup, sampler)
-        tbps = world * n * bits / (ms * 1e-3) / 1e12
+        tbps = n_total * bits / (ms * 1e-3) / 1e12
         res = {"value": tbps, "ms_per_step": ms, "kernel_ms_per_step": kms,
                "kernel_tbps_per_gpu": n * bits / (kms * 1e-3) / 1e12,
                "gpu_launches": launches, "roofline": roofline(kms, clocks)}
@@ -304,10 +360,7 @@ def run_ours(args, rank, world, local_rank):
     # checksum of one consume step (sharding invariant), outside the timed region
     step_consume()
     torch.cuda.synchronize(dev)
-    cs = cs_out.clone()
-    if world > 1:
-        dist.all_reduce(cs, op=dist.ReduceOp.SUM)
-    checksum = int(cs.item()) & ((1 << 64) - 1)
+    checksum = shard.allreduce_checksum(int(cs_out.item()), device=dev)
 
     # e2e: host keys (pinned) -> rekey through the C ABI -> CHECKSUM -> 8 B back to host
     e2e = None
@@ -325,18 +378,16 @@ def run_ours(args, rank, world, local_rank):
                 cs_host.copy_(cs_out, non_blocking=True)
 
         ms_e2e, _, _, _ = timed(step_e2e, max(1, args.steps), 1)
-        e2e = {"value": world * n * bits / (ms_e2e * 1e-3) / 1e12, "unit": "Tb/s",
+        e2e = {"value": n_total * bits / (ms_e2e * 1e-3) / 1e12, "unit": "Tb/s",
                "h2d_bytes_per_step": int(keys_h.nbytes + ivs_h.nbytes), "d2h_bytes_per_step": 8,
                "ms_per_step": ms_e2e, "mode": "consume"}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        cores = cpu_cores()
-        n_s, bits_s = 8 * cores, 1 << 16
-        r, dt = oracle_sample(n_s, bits_s, threads=cores)
-        cpu = {"value": r / 1e12, "unit": "Tb/s", "cores": cores, "kind": "oracle",
-               "sample": f"{n_s} instances x {bits_s} bits ({dt:.1f} s), first instances of the workload, "
-                         f"{cpu_model()}", "bits_per_s_per_core": r / cores}
+        cpu = cpu_baseline()
+    context = None
+    if rank == 0 and world == 1 and not args.no_context:
+        context = run_context(local_rank)
 
     if rank == 0:
         head = results[args.mode]
@@ -348,14 +399,14 @@ def run_ours(args, rank, world, local_rank):
         line = {
             "metric": METRIC, "value": head["value"], "unit": "Tb/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": head["ms_per_step"],
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
+            "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "u32",
             "data": "synthetic (SplitMix64 keys/IVs, seed 0x5EED2020)",
-            "config": {"workload": f"configs[1]: MICKEY 2.0, {n} instances x {bits} bits per GPU per step "
-                                   f"({args.mode})", "instances_per_gpu": n, "bits_per_instance": bits,
+            "config": {"workload": f"{desc} ({args.mode})", "instances_total": n_total,
+                       "instances_per_gpu": n, "bits_per_instance": bits,
                        "mode": args.mode, "parallelism": f"instance-range shards x{world}",
                        "l2": "flushed (256 MiB write) between timed steps; state 100 MiB, keys 80 MiB"},
             "roofline": rf, "clocks": head.get("clocks"), "gpu_launches": head["gpu_launches"],
-            "e2e": e2e, "cpu_baseline": cpu, "checksum": f"{checksum:016x}",
+            "e2e": e2e, "cpu_baseline": cpu, "checksum": f"{checksum:016x}", "context": context,
             "modes": {m: {k: v for k, v in r.items() if k != "clocks"} for m, r in results.items()},
             "paper_context": "2.72 Tb/s RTX 2080 Ti, 2.90 Tb/s V100 (PAPER.md:46-50, 852-854); "
                              "exceeds the bit-exact LOP3 bound on those GPUs, see BASELINE.md",

@@ -73,7 +73,7 @@ struct bsrng {
     uint32_t* state = nullptr;   // [NSTATE + 1][Gp]
     uint32_t* sliced = nullptr;  // key [KB][Gp] then iv [IVB][Gp]
     uint8_t* raw = nullptr;      // keys [n][key_bytes] then ivs [n][iv_bytes]
-    uint32_t* sched = nullptr;   // [1 + units]: ticket, flags
+    uint32_t* sched = nullptr;   // [1 + units]: ticket, flags; then [32] scratch
     uint8_t* bounce = nullptr;   // generate_host staging
     uint64_t bounce_bytes = 0;
     // options
@@ -164,7 +164,13 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
     a.out = out;
     a.row_bytes = bits / 8;
     a.units = h->units;
+    a.scratch = h->sched + 1 + h->units;
 
+    const size_t smem = LAYOUT == bsk::L_ROW_MAJOR ? size_t(KS_BLOCK / 32) * bsk::RM_WARP_WORDS * 4 : 0;
+    if (smem > 48 * 1024) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+        if (e != cudaSuccess) return fail(BSRNG_ECUDA, "smem attribute: %s", cudaGetErrorString(e));
+    }
     unsigned grid;
     if (h->opt_sched == 0) {
         a.persistent = 0;
@@ -172,11 +178,11 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
         a.seg_clocks = bits;
         grid = unsigned((h->Gp + KS_BLOCK - 1) / KS_BLOCK);
     } else {
-        int occ = h->opt_ctas_per_sm;
-        if (occ <= 0) {
-            if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, KS_BLOCK, 0) != cudaSuccess || occ < 1)
-                occ = 1;
-        }
+        int occ = h->opt_ctas_per_sm, occ_max = 1;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_max, kern, KS_BLOCK, smem) != cudaSuccess ||
+            occ_max < 1)
+            occ_max = 1;
+        if (occ <= 0 || occ > occ_max) occ = occ_max;
         const uint64_t slots = uint64_t(h->num_sms) * occ * (KS_BLOCK / 32);  // resident warps
         uint64_t nseg = 1;
         if (h->opt_seg_clocks) {
@@ -187,7 +193,9 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
             nseg = std::max<uint64_t>(1, (32 * slots + h->units - 1) / h->units);
             nseg = std::min<uint64_t>(nseg, std::max<uint64_t>(1, bits / 256));
         }
-        uint64_t seg = ((bits + nseg - 1) / nseg + 31) / 32 * 32;
+        // whole 256-clock blocks keep ROW_MAJOR sector flushes full (32 B/row)
+        const uint64_t quantum = bits >= 256 ? 256 : 32;
+        uint64_t seg = ((bits + nseg - 1) / nseg + quantum - 1) / quantum * quantum;
         nseg = (bits + seg - 1) / seg;
         a.persistent = 1;
         a.nseg = nseg;
@@ -211,7 +219,7 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
         cudaMemsetAsync(dbg, 0, 4 * sizeof(unsigned long long), st);
         a.dbg = dbg;
     }
-    kern<<<grid, KS_BLOCK, 0, st>>>(a);
+    kern<<<grid, KS_BLOCK, smem, st>>>(a);
     int rc = check_launch("keystream");
     if (dbg) {
         unsigned long long c[4];
@@ -300,7 +308,7 @@ bsrng_t* bsrng_create_ex(bsrng_cipher cipher, const uint8_t* keys, const uint8_t
     if (cudaMalloc(&h->state, uint64_t(ns + 1) * h->Gp * 4) != cudaSuccess ||
         cudaMalloc(&h->sliced, sl_words * 4) != cudaSuccess ||
         cudaMalloc(&h->raw, h->n * (h->key_bytes + h->iv_bytes)) != cudaSuccess ||
-        cudaMalloc(&h->sched, (1 + h->units) * 4) != cudaSuccess) {
+        cudaMalloc(&h->sched, (1 + h->units + 32) * 4) != cudaSuccess) {
         cudaGetLastError();
         bsrng_destroy(h);
         fail(BSRNG_ENOMEM, "cudaMalloc failed for %llu instances", (unsigned long long)n);

@@ -50,6 +50,7 @@ struct KsArgs {
     uint64_t units;       // warp-units = Gp / 32
     uint32_t* ticket;     // persistent mode: [1], zeroed before launch
     uint32_t* flags;      // persistent mode: [units], zeroed before launch
+    uint32_t* scratch;    // [32] sink for padding-group SLICED stores
     unsigned long long* dbg;  // optional scheduler counters (BSRNG_DEBUG), or null
     int persistent;
 };
@@ -70,14 +71,23 @@ __device__ __forceinline__ uint32_t lane_mask(const KsArgs& a, uint64_t g)
     return g + 1 < a.G ? 0xFFFFFFFFu : (g + 1 == a.G ? a.tail_mask : 0u);
 }
 
-// Transpose the 32 staged slice words zs[t][lane] (t = 0..31) of this thread
-// and store its instance rows.  Row t of the bit matrix is clock t, or clock
-// t^7 for MSB-first ciphers so that clock 8b+q lands in bit 7-q of byte b.
-//   row0  : address of (instance 32g, this 32-clock block) in the output
-//   nvalid: rows of this group that are real instances (0..32)
+// ROW_MAJOR staging per warp (dynamic shared memory):
+//   zs: z words of the current 32-clock block, [t][lane]      (4 KB / warp)
+//   os: transposed words for one 32-byte sector of every row,
+//       [row q][slot k][lane], k = 32-clock block within the sector (32 KB)
+// Every access is lane-contiguous, so STS/LDS are bank-conflict free.  Rows are
+// written as whole 32 B sectors (two 16 B stores): 4-byte stores spread over
+// the ~600k rows in flight overflowed L2 before their sectors filled, and the
+// partial-sector evictions cost ~15x the algorithmic DRAM traffic (ncu).
+constexpr int ZS_WORDS = 32 * 32;
+constexpr int OS_WORDS = 32 * 8 * 32;
+constexpr int RM_WARP_WORDS = ZS_WORDS + OS_WORDS;
+
+// Transpose this thread's 32 staged z words (a 32x32 bit block) and park the
+// 32 row words in sector slot `k`.  Bit-matrix row t is clock t, or clock t^7
+// for MSB-first ciphers so that clock 8b+q lands in bit 7-q of byte b.
 template <bool MSB_FIRST>
-__device__ __forceinline__ void rowmajor_flush(const uint32_t* zs, uint8_t* row0, uint64_t row_bytes,
-                                               uint32_t nvalid)
+__device__ __forceinline__ void rowmajor_transpose(const uint32_t* zs, uint32_t* os, uint32_t k)
 {
     constexpr int X = MSB_FIRST ? 7 : 0;
 #pragma unroll
@@ -85,15 +95,36 @@ __device__ __forceinline__ void rowmajor_flush(const uint32_t* zs, uint8_t* row0
         uint32_t x[16];
 #pragma unroll
         for (int q = 0; q < 16; ++q) {
-            const uint32_t lo = zs[((q ^ X)) * 32];
+            const uint32_t lo = zs[(q ^ X) * 32];
             const uint32_t hi = zs[((q + 16) ^ X) * 32];
             x[q] = __byte_perm(lo, hi, h == 0 ? 0x5410 : 0x7632);
         }
         bt_transpose16(x);
 #pragma unroll
-        for (int q = 0; q < 16; ++q)
-            if (uint32_t(16 * h + q) < nvalid)
-                *reinterpret_cast<uint32_t*>(row0 + uint64_t(16 * h + q) * row_bytes) = x[q];
+        for (int q = 0; q < 16; ++q) os[((16 * h + q) * 8 + k) * 32] = x[q];
+    }
+}
+
+// Write slots [k_lo, k_hi] of every real row of this thread's group.
+//   row0: address of instance 32g's row; col: byte column of slot k_lo.
+__device__ __forceinline__ void rowmajor_store(const uint32_t* os, uint8_t* row0, uint64_t row_bytes,
+                                               uint32_t nvalid, uint32_t k_lo, uint32_t k_hi, uint64_t col)
+{
+    uint8_t* p = row0 + col;
+    if (k_lo == 0 && k_hi == 7 && ((reinterpret_cast<uintptr_t>(p) | row_bytes) & 15) == 0) {
+#pragma unroll 4
+        for (uint32_t q = 0; q < nvalid; ++q) {
+            const uint32_t* src = os + q * 8 * 32;
+            const uint4 v0 = make_uint4(src[0], src[32], src[64], src[96]);
+            const uint4 v1 = make_uint4(src[128], src[160], src[192], src[224]);
+            uint4* d = reinterpret_cast<uint4*>(p + q * row_bytes);
+            __stcs(d, v0);
+            __stcs(d + 1, v1);
+        }
+    } else {
+        for (uint32_t q = 0; q < nvalid; ++q)
+            for (uint32_t k = k_lo; k <= k_hi; ++k)
+                __stcs(reinterpret_cast<uint32_t*>(p + q * row_bytes + (k - k_lo) * 4), os[(q * 8 + k) * 32]);
     }
 }
 
@@ -117,7 +148,9 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
 {
     static_assert(32 % U == 0, "U must divide 32");
     constexpr int NW = BLOCK / 32;
-    __shared__ uint32_t zs_all[LAYOUT == L_ROW_MAJOR ? NW * 32 * 32 : 1];
+    extern __shared__ uint32_t rm_smem[];  // ROW_MAJOR only: NW * RM_WARP_WORDS
+    __shared__ uint8_t* s_row0[LAYOUT == L_ROW_MAJOR ? BLOCK : 1];
+    __shared__ uint32_t s_nvalid[LAYOUT == L_ROW_MAJOR ? BLOCK : 1];
     __shared__ uint32_t s_item[NW];
     // Only `s_item` (smem) and the loop counters survive a clock loop; every
     // other per-item value is re-derived afterwards, so the 200 state words
@@ -174,14 +207,15 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
             }
         } else if (LAYOUT == L_SLICED) {
             const uint32_t m = lane_mask(a, g);
-            uint32_t* o = static_cast<uint32_t*>(a.out) + clk_begin * a.G + (g < a.G ? g : 0);
-            const uint64_t stride = g < a.G ? a.G : 0;  // 0 = padding group: never stores
+            // padding groups (g >= G) write to a private scratch word instead of
+            // being predicated off, so the loop body has no branches
+            uint32_t* o = g < a.G ? static_cast<uint32_t*>(a.out) + clk_begin * a.G + g : a.scratch + lane;
+            const uint64_t stride = g < a.G ? a.G : 0;
 #pragma unroll 1
             for (uint32_t it = nclk / U; it != 0; --it) {
 #pragma unroll
                 for (int u = 0; u < U; ++u) {
-                    const uint32_t z = c.z() & m;
-                    if (stride) __stcs(o, z);
+                    __stcs(o, c.z() & m);
                     o += stride;
                     c.clock();
                 }
@@ -189,10 +223,13 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
         } else {  // ROW_MAJOR
             const uint64_t first = g * 32u;
             const uint32_t nvalid = first >= a.n ? 0u : uint32_t(a.n - first < 32 ? a.n - first : 32);
-            uint8_t* row0 = static_cast<uint8_t*>(a.out) + (nvalid ? first : 0) * a.row_bytes + (clk_begin >> 3);
-            uint32_t* zs = zs_all + (threadIdx.x >> 5) * 32 * 32 + lane;
+            s_row0[threadIdx.x] = static_cast<uint8_t*>(a.out) + (nvalid ? first : 0) * a.row_bytes;
+            s_nvalid[threadIdx.x] = nvalid;
+            uint32_t* zs = rm_smem + (threadIdx.x >> 5) * RM_WARP_WORDS + lane;
+            const uint64_t b0 = clk_begin >> 5;  // call-relative index of the first 32-clock block
+            const uint32_t nblk = nclk >> 5;
 #pragma unroll 1
-            for (uint32_t blk = nclk / 32; blk != 0; --blk) {
+            for (uint32_t blk = 0; blk < nblk; ++blk) {
 #pragma unroll 1
                 for (uint32_t k = 0; k < 32; k += U) {
 #pragma unroll
@@ -201,8 +238,14 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
                         c.clock();
                     }
                 }
-                rowmajor_flush<C::MSB_FIRST>(zs, row0, a.row_bytes, nvalid);
-                row0 += 4;
+                const uint64_t B = b0 + blk;
+                const uint32_t k = uint32_t(B & 7);
+                rowmajor_transpose<C::MSB_FIRST>(zs, zs + ZS_WORDS, k);
+                if (k == 7 || blk + 1 == nblk) {
+                    const uint32_t k_lo = k - (blk < k ? blk : k);
+                    rowmajor_store(zs + ZS_WORDS, s_row0[threadIdx.x], a.row_bytes, s_nvalid[threadIdx.x], k_lo,
+                                   k, (B - (k - k_lo)) * 4);
+                }
             }
         }
 

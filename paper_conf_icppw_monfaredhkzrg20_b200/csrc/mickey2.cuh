@@ -16,6 +16,7 @@
 // control 1, output 1 = 327 LOP3 for 32 keystream bits.
 #pragma once
 #include <cstdint>
+#include <utility>
 
 #include "bitslice.cuh"
 
@@ -46,7 +47,39 @@ __device__ __forceinline__ uint32_t lop3(uint32_t a, uint32_t b, uint32_t c)
     uint32_t d;
     asm("lop3.b32 %0, %1, %2, %3, %4;" : "=r"(d) : "r"(a), "r"(b), "r"(c), "n"(LUT));
     return d;
-}  // slice words of state per group: r_0..r_99, s_0..s_99
+}
+
+// s'_I = s^_I ^ (feedback term of category (FB0_I, FB1_I)).  s^_I is one LOP3
+// whose truth table folds COMP0_I / COMP1_I in at compile time (explicit PTX:
+// left to itself ptxas keeps some s_i complemented and pays NOTs for them).
+template <int I>
+__device__ __forceinline__ uint32_t s_next(const uint32_t (&s)[100], uint32_t fb_s, uint32_t fb_s0, uint32_t fb_s1)
+{
+    uint32_t v;
+    if constexpr (I == 0) {
+        v = 0u;
+    } else if constexpr (I == 99) {
+        v = s[98];
+    } else {
+        constexpr uint32_t c0 = comp0(I) & 0xFFu, c1 = comp1(I) & 0xFFu;
+        constexpr uint32_t LUT = 0xF0u ^ ((0xCCu ^ c0) & (0xAAu ^ c1));
+        v = lop3<LUT>(s[I - 1], s[I], s[I + 1]);
+    }
+    if constexpr (fb0(I) && fb1(I))
+        v = (I == 0) ? fb_s : (v ^ fb_s);
+    else if constexpr (fb0(I))
+        v ^= fb_s0;
+    else if constexpr (fb1(I))
+        v ^= fb_s1;
+    return v;
+}
+
+template <int... I>
+__device__ __forceinline__ void s_update(uint32_t (&ns)[100], const uint32_t (&s)[100], uint32_t fb_s, uint32_t fb_s0,
+                                         uint32_t fb_s1, std::integer_sequence<int, I...>)
+{
+    ((ns[I] = s_next<I>(s, fb_s, fb_s0, fb_s1)), ...);
+}
 
 // One CLOCK_KG on 32 lanes.  MIX = the spec's MIXING flag (init clocks);
 // `in` = INPUT_BIT slice word (ignored unless MIX).
@@ -76,23 +109,7 @@ __device__ __forceinline__ void clock_kg(uint32_t (&r)[100], uint32_t (&s)[100],
     r[0] = lop3<LUT_A_XOR_BC>(fb_r, ctl_r, r[0]);  // 0 is in RTAPS
 
     uint32_t ns[100];
-#pragma unroll
-    for (int i = 0; i < 100; ++i) {
-        uint32_t v;
-        if (i == 0)
-            v = 0u;
-        else if (i == 99)
-            v = s[98];
-        else
-            v = s[i - 1] ^ ((s[i] ^ comp0(i)) & (s[i + 1] ^ comp1(i)));
-        if (fb0(i) && fb1(i))
-            v ^= fb_s;
-        else if (fb0(i))
-            v ^= fb_s0;
-        else if (fb1(i))
-            v ^= fb_s1;
-        ns[i] = v;
-    }
+    s_update(ns, s, fb_s, fb_s0, fb_s1, std::make_integer_sequence<int, 100>{});
 #pragma unroll
     for (int i = 0; i < 100; ++i) s[i] = ns[i];
 }
