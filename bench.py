@@ -161,7 +161,7 @@ def oracle_sample(n_inst, bits, first=0, threads=None):
     return n_inst * bits / dt, dt
 
 
-def cpu_baseline(target_s=12.0):
+def cpu_baseline(target_s=25.0):
     """The oracle as it stands, on all host cores, on a bounded sample of the
     workload (its first instances, 2^16 bits each) sized for ~target_s."""
     cores = cpu_cores()
@@ -213,7 +213,7 @@ def run_reference(args, rank, world):
         return
     _, _, scaling, desc = workload(args, world)
     cores = cpu_cores()
-    n_s, bits_s = 16 * cores, 1 << 15
+    n_s, bits_s = 64 * cores, 1 << 15
     for _ in range(args.warmup):
         oracle_sample(n_s, bits_s, threads=cores)
     tot_bits, tot_t = 0, 0.0
