@@ -19,7 +19,7 @@ from concurrent.futures import ThreadPoolExecutor
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-_SOURCES = ["mickey2_ref.c"]
+_SOURCES = ["mickey2_ref.c", "grain_ref.c"]
 _LIB_PATH = os.path.join(_HERE, "liboracle.so")
 _lib = None
 
@@ -51,6 +51,12 @@ def lib() -> ctypes.CDLL:
         L.ref_mickey2_clock_kg.restype = None
         L.ref_mickey2_table.argtypes = [ctypes.c_int, ctypes.c_int]
         L.ref_mickey2_table.restype = ctypes.c_int
+        L.ref_grain_keystream.argtypes = [u8p, u8p, ctypes.c_uint64, u8p]
+        L.ref_grain_keystream.restype = None
+        L.ref_grain_state.argtypes = [u8p, u8p, ctypes.c_uint64, u8p, u8p]
+        L.ref_grain_state.restype = None
+        L.ref_grain_clock.argtypes = [u8p, u8p, ctypes.c_int]
+        L.ref_grain_clock.restype = ctypes.c_int
         _lib = L
     return _lib
 
@@ -123,6 +129,55 @@ def mickey2_keystream_batch(keys: np.ndarray, ivs: np.ndarray, iv_bits: int, nbi
         rc = L.ref_mickey2_keystream(_p(keys[i]), _p(ivpad[i]), iv_bits, nbits, _p(out[i]))
         if rc != 0:
             raise ValueError("bad iv_bits")
+
+    threads = threads or os.cpu_count() or 1
+    if threads == 1 or n == 1:
+        for i in range(n):
+            one(i)
+    else:
+        with ThreadPoolExecutor(max_workers=threads) as ex:
+            list(ex.map(one, range(n)))
+    return out[:, :nbytes]
+
+
+# -------------------------------------------------------------------- Grain v1
+def grain_keystream(key: bytes, iv: bytes, nbits: int) -> bytes:
+    """Grain v1 keystream of one instance, packed LSB-first."""
+    k = _buf(key, 10)
+    v = _buf(iv, 8)
+    out = np.zeros(max((nbits + 7) // 8, 1), dtype=np.uint8)
+    lib().ref_grain_keystream(_p(k), _p(v), nbits, _p(out))
+    return out[: (nbits + 7) // 8].tobytes()
+
+
+def grain_state(key: bytes, iv: bytes, extra_clocks: int = 0):
+    """(s, b) = (LFSR, NFSR) as uint8[80] 0/1 arrays after init (+ clocks)."""
+    k = _buf(key, 10)
+    v = _buf(iv, 8)
+    s = np.zeros(80, dtype=np.uint8)
+    b = np.zeros(80, dtype=np.uint8)
+    lib().ref_grain_state(_p(k), _p(v), extra_clocks, _p(s), _p(b))
+    return s, b
+
+
+def grain_clock(s: np.ndarray, b: np.ndarray, init_mode: int):
+    s = np.ascontiguousarray(s, dtype=np.uint8).copy()
+    b = np.ascontiguousarray(b, dtype=np.uint8).copy()
+    z = lib().ref_grain_clock(_p(s), _p(b), int(init_mode))
+    return s, b, z
+
+
+def grain_keystream_batch(keys: np.ndarray, ivs: np.ndarray, nbits: int, threads: int | None = None):
+    """Row-major Grain keystreams, uint8[n, ceil(nbits/8)] (LSB-first)."""
+    keys = np.ascontiguousarray(keys, dtype=np.uint8)
+    ivs = np.ascontiguousarray(ivs, dtype=np.uint8)
+    n = keys.shape[0]
+    nbytes = (nbits + 7) // 8
+    out = np.zeros((n, max(nbytes, 1)), dtype=np.uint8)
+    L = lib()
+
+    def one(i):
+        L.ref_grain_keystream(_p(keys[i]), _p(ivs[i]), nbits, _p(out[i]))
 
     threads = threads or os.cpu_count() or 1
     if threads == 1 or n == 1:
