@@ -143,7 +143,9 @@ uint64_t bsrng_bits_done(const bsrng_t* h);
 /*
  * bsrng_copy_state -- copy the sliced cipher state to HOST memory (synchronous):
  * MICKEY: uint32[200][G] (rows 0..99 = R bits r_0..r_99, rows 100..199 = S
- * bits s_0..s_99; bit j of word [i][g] = that bit of instance 32g+j).
+ * bits s_0..s_99); Grain v1: uint32[160][G] (rows 0..79 = LFSR s_0..s_79,
+ * rows 80..159 = NFSR b_0..b_79).  Bit j of word [i][g] = that bit of
+ * instance 32g+j.
  * `words` is the capacity of host_out in uint32 words.  Returns the number of
  * words written (>0) or a negative error code.
  */

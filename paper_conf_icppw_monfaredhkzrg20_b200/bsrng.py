@@ -23,7 +23,7 @@ OK, EINVAL, ENOMEM, ECUDA, ERANGE, EUNSUPPORTED = 0, -1, -2, -3, -4, -5
 
 CIPHERS = {"mickey2": MICKEY2, "grain": GRAIN_V1, "aes128ctr": AES128_CTR}
 LAYOUTS = {"row_major": ROW_MAJOR, "sliced": SLICED, "checksum": CHECKSUM}
-NSTATE = {MICKEY2: 200}
+NSTATE = {MICKEY2: 200, GRAIN_V1: 160}
 DEFAULT_IV_BITS = {MICKEY2: 80, GRAIN_V1: 64, AES128_CTR: 128}
 
 SYMBOLS = [

@@ -1,0 +1,152 @@
+// grain.cuh -- bitsliced Grain v1 for sm_100a.
+//
+// PAPER.md:339-357 (sec. 2.3.3, Fig. 4): Grain, an 80-bit LFSR s and an 80-bit
+// NFSR b, LFSR feedback f, NFSR feedback g, filter h; 80-bit key, 64-bit IV,
+// 160 initialisation clocks; PAPER.md:456-460 and Fig. 10: the paper's second
+// bitsliced stream cipher.  Definitions follow the Grain v1 specification
+// (ref [15]).  One thread = 32 instances; every register bit
+// is a 32-lane slice word.
+//
+// Both registers shift by one position per clock (Fibonacci form), so the
+// shift is pure register renaming; only the three new words (f, g, z) cost
+// logic: ~39 LOP3 per clock per 32 keystream bits, 8x cheaper
+// than MICKEY 2.0.  The renaming closes every 80 clocks; with U clocks per loop
+// iteration ptxas restores the register map at the back edge with moves
+// (160/U per clock, issued on the otherwise idle FMA pipe).
+#pragma once
+#include <cstdint>
+
+#include "bitslice.cuh"
+
+namespace bsk {
+namespace grain {
+
+constexpr int NSTATE = 160;  // s_0..s_79, b_0..b_79
+
+// h(x0..x4) = x1+x4+x0x3+x2x3+x3x4+x0x1x2+x0x2x3+x0x2x4+x1x2x4+x2x3x4
+//           = [x1 + x4 + x3(x0 + x4)] + x2 [x3 + x0x1 + x0x3 + x0x4 + x1x4 + x3x4]
+__device__ __forceinline__ uint32_t h_filter(uint32_t x0, uint32_t x1, uint32_t x2, uint32_t x3, uint32_t x4)
+{
+    const uint32_t a = x1 ^ x4 ^ (x3 & (x0 ^ x4));
+    const uint32_t b = x3 ^ (x0 & x1) ^ (x0 & x3) ^ (x0 & x4) ^ (x1 & x4) ^ (x3 & x4);
+    return a ^ (x2 & b);
+}
+
+// z = b1+b2+b4+b10+b31+b43+b56 + h(s3, s25, s46, s64, b63)
+__device__ __forceinline__ uint32_t output(const uint32_t (&s)[80], const uint32_t (&b)[80])
+{
+    return b[1] ^ b[2] ^ b[4] ^ b[10] ^ b[31] ^ b[43] ^ b[56] ^ h_filter(s[3], s[25], s[46], s[64], b[63]);
+}
+
+// f: s_80 = s62+s51+s38+s23+s13+s0
+__device__ __forceinline__ uint32_t f_lfsr(const uint32_t (&s)[80])
+{
+    return s[62] ^ s[51] ^ s[38] ^ s[23] ^ s[13] ^ s[0];
+}
+
+// g: b_80 = s0 + b62+b60+b52+b45+b37+b33+b28+b21+b14+b9+b0 + b63b60 + b37b33 + b15b9
+//         + b60b52b45 + b33b28b21 + b63b45b28b9 + b60b52b37b33 + b63b60b21b15
+//         + b63b60b52b45b37 + b33b28b21b15b9 + b52b45b37b33b28b21
+// with the shared products p60_63, p33_37, p9_15, p45_52, p21_28.
+__device__ __forceinline__ uint32_t g_nfsr(uint32_t s0, const uint32_t (&b)[80])
+{
+    const uint32_t p60_63 = b[63] & b[60];
+    const uint32_t p33_37 = b[37] & b[33];
+    const uint32_t p9_15 = b[15] & b[9];
+    const uint32_t p45_52 = b[52] & b[45];
+    const uint32_t p21_28 = b[28] & b[21];
+    const uint32_t p21_28_33 = p21_28 & b[33];
+    uint32_t v = s0 ^ b[62] ^ b[60] ^ b[52] ^ b[45] ^ b[37] ^ b[33] ^ b[28] ^ b[21] ^ b[14] ^ b[9] ^ b[0];
+    v ^= p60_63 ^ p33_37 ^ p9_15;
+    v ^= b[60] & p45_52;
+    v ^= p21_28_33;
+    v ^= (b[63] & b[45]) & (b[28] & b[9]);
+    v ^= b[60] & b[52] & p33_37;
+    v ^= p60_63 & b[21] & b[15];
+    v ^= p60_63 & p45_52 & b[37];
+    v ^= p21_28_33 & p9_15;
+    v ^= p45_52 & p33_37 & p21_28;
+    return v;
+}
+
+// One clock.  INIT = the initialisation mode: z is added to both feedbacks.
+template <bool INIT>
+__device__ __forceinline__ void clock(uint32_t (&s)[80], uint32_t (&b)[80])
+{
+    uint32_t fs = f_lfsr(s);
+    uint32_t fb = g_nfsr(s[0], b);
+    if (INIT) {
+        const uint32_t z = output(s, b);
+        fs ^= z;
+        fb ^= z;
+    }
+#pragma unroll
+    for (int i = 0; i < 79; ++i) {
+        s[i] = s[i + 1];
+        b[i] = b[i + 1];
+    }
+    s[79] = fs;
+    b[79] = fb;
+}
+
+}  // namespace grain
+
+// Cipher traits used by keystream_kernel (keystream.cuh).
+struct Grain {
+    static constexpr int NSTATE = grain::NSTATE;
+    static constexpr bool MSB_FIRST = false;  // spec [15]: keystream packed LSB-first
+    // clocks per loop iteration (~45 instructions per clock).  The 80-clock
+    // register rotation costs 160/U moves per clock at the back edge; at U = 32
+    // ptxas emits them all as IMAD.MOV (FMA pipe), at U = 16 partly as MOV.
+    static constexpr int U_DEFAULT = 32, U_ALT0 = 8, U_ALT1 = 16;
+    uint32_t s[80], b[80];
+
+    __device__ __forceinline__ void load(const uint32_t* st, uint64_t Gp, uint64_t g)
+    {
+        const uint32_t* p = opaque(st + g);
+#pragma unroll
+        for (int i = 0; i < 80; ++i) s[i] = __ldcg(p + uint64_t(i) * Gp);
+#pragma unroll
+        for (int i = 0; i < 80; ++i) b[i] = __ldcg(p + uint64_t(80 + i) * Gp);
+    }
+    __device__ __forceinline__ void store(uint32_t* st, uint64_t Gp, uint64_t g) const
+    {
+        uint32_t* p = opaque(st + g);
+#pragma unroll
+        for (int i = 0; i < 80; ++i) __stcg(p + uint64_t(i) * Gp, s[i]);
+#pragma unroll
+        for (int i = 0; i < 80; ++i) __stcg(p + uint64_t(80 + i) * Gp, b[i]);
+    }
+    __device__ __forceinline__ uint32_t z() const { return grain::output(s, b); }
+    __device__ __forceinline__ void clock() { grain::clock<false>(s, b); }
+};
+
+// Initialisation (spec [15]): b_i = key bit i, s_i = IV bit i (i < 64),
+// s_64..s_79 = 1, then 160 clocks with z fed back.  Key/IV bits LSB-first.
+//   key_s: uint32 [80][Gp], iv_s: uint32 [64][Gp]; state uint32 [161][Gp].
+__global__ void __launch_bounds__(128) grain_preclock_kernel(const uint32_t* __restrict__ key_s,
+                                                             const uint32_t* __restrict__ iv_s,
+                                                             uint32_t* __restrict__ state, uint64_t Gp)
+{
+    const uint64_t g = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (g >= Gp) return;
+    uint32_t s[80], b[80];
+#pragma unroll
+    for (int i = 0; i < 80; ++i) b[i] = key_s[uint64_t(i) * Gp + g];
+#pragma unroll
+    for (int i = 0; i < 64; ++i) s[i] = iv_s[uint64_t(i) * Gp + g];
+#pragma unroll
+    for (int i = 64; i < 80; ++i) s[i] = 0xFFFFFFFFu;
+#pragma unroll 1
+    for (int c = 0; c < 160; c += 16) {
+#pragma unroll
+        for (int u = 0; u < 16; ++u) grain::clock<true>(s, b);
+    }
+#pragma unroll
+    for (int i = 0; i < 80; ++i) state[uint64_t(i) * Gp + g] = s[i];
+#pragma unroll
+    for (int i = 0; i < 80; ++i) state[uint64_t(80 + i) * Gp + g] = b[i];
+    state[uint64_t(160) * Gp + g] = 0u;
+}
+
+}  // namespace bsk

@@ -123,6 +123,9 @@ namespace bsk {
 struct Mickey2 {
     static constexpr int NSTATE = m2::NSTATE;
     static constexpr bool MSB_FIRST = true;  // spec [5]: keystream packed MSB-first
+    // clocks per loop iteration: 4 keeps the loop (21 KB of SASS) in the
+    // instruction cache; 2 and 8 are built for sweeps ("unroll" option)
+    static constexpr int U_DEFAULT = 4, U_ALT0 = 2, U_ALT1 = 8;
     uint32_t r[100], s[100];
 
     // State carry (SURVEY step a-5).  The row pointer goes through opaque()
