@@ -34,9 +34,16 @@ sys.path.insert(0, ROOT)
 
 N_DEFAULT = 1 << 22
 BITS_DEFAULT = 1 << 20
-LOP3_PER_CLOCK = 327           # DESIGN.md / SURVEY App. D: algorithmic ops per clock per group
+# algorithmic LOP3 per clock per 32-instance group
+LOP3_PER_CLOCK = {"mickey2": 327, "grain": 39}
+CIPHER_NAME = {"mickey2": "MICKEY 2.0", "grain": "Grain v1"}
 ALU_LANES_PER_SM_CLK = 64      # 4 SMSP x 16 lanes (alu pipe rt = 2 cycles/warp-instr)
 METRIC = "MICKEY 2.0 keystream Tb/s (1 and 8 B200); fraction of LOP3/HBM roofline"
+
+
+def metric(args):
+    """BASELINE.json's metric; with --cipher grain the same metric for Grain v1 (configs[3])."""
+    return METRIC if args.cipher == "mickey2" else METRIC.replace("MICKEY 2.0", CIPHER_NAME[args.cipher])
 
 
 def parse():
@@ -45,9 +52,11 @@ def parse():
     p.add_argument("--steps", type=int, default=3)
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    p.add_argument("--workload", default="c2", choices=["c2", "c3"],
+    p.add_argument("--workload", default="c2", choices=["c2", "c3", "c4"],
                    help="c2 = BASELINE configs[1] per GPU (weak scaling); "
-                        "c3 = configs[2]: 2^25 instances x 2^18 bits = 1 TiB total, split across GPUs (strong)")
+                        "c3 = configs[2]: 2^25 instances x 2^18 bits = 1 TiB total, split across GPUs (strong); "
+                        "c4 = configs[3]: the paper's launch shape, 2^19 instances x 4416 clocks per GPU")
+    p.add_argument("--cipher", default="mickey2", choices=["mickey2", "grain"])
     p.add_argument("--n", type=int, default=None, help="instances per GPU (c2) / in total (c3)")
     p.add_argument("--bits", type=int, default=None, help="keystream bits per instance per step")
     p.add_argument("--no-context", action="store_true", help="skip the ALU-peak / cuRAND microbenchmarks")
@@ -150,25 +159,28 @@ def cpu_model():
     return "unknown"
 
 
-def oracle_sample(n_inst, bits, first=0, threads=None):
+def oracle_sample(n_inst, bits, first=0, threads=None, cipher="mickey2"):
     """Time the oracle (unmodified, bit-serial) on host cores; returns bits/s."""
     import oracle
     from paper_conf_icppw_monfaredhkzrg20_b200 import inputs
-    keys, ivs = inputs.make_inputs("mickey2", n_inst, first)
+    keys, ivs = inputs.make_inputs(cipher, n_inst, first)
     t = time.perf_counter()
-    oracle.mickey2_keystream_batch(keys, ivs, 80, bits, threads=threads)
+    if cipher == "grain":
+        oracle.grain_keystream_batch(keys, ivs, bits, threads=threads)
+    else:
+        oracle.mickey2_keystream_batch(keys, ivs, 80, bits, threads=threads)
     dt = time.perf_counter() - t
     return n_inst * bits / dt, dt
 
 
-def cpu_baseline(target_s=25.0):
+def cpu_baseline(target_s=25.0, cipher="mickey2"):
     """The oracle as it stands, on all host cores, on a bounded sample of the
     workload (its first instances, 2^16 bits each) sized for ~target_s."""
     cores = cpu_cores()
-    r0, _ = oracle_sample(2 * cores, 1 << 13, threads=cores)      # calibration
+    r0, _ = oracle_sample(2 * cores, 1 << 13, threads=cores, cipher=cipher)  # calibration
     n_s = int(max(cores, min(1 << 16, r0 * target_s / (1 << 16))))
     n_s = (n_s + cores - 1) // cores * cores
-    r, dt = oracle_sample(n_s, 1 << 16, threads=cores)
+    r, dt = oracle_sample(n_s, 1 << 16, threads=cores, cipher=cipher)
     return {"value": r / 1e12, "unit": "Tb/s", "cores": cores, "kind": "oracle",
             "sample": f"instances 0..{n_s - 1} of the workload x 65536 bits ({dt:.1f} s), {cpu_model()}",
             "bits_per_s_per_core": r / cores}
@@ -198,13 +210,19 @@ def run_context(local_rank):
 # ------------------------------------------------------------ reference arm
 def workload(args, world):
     """(n_total, bits, scaling, description) of the benchmarked configuration."""
+    name = CIPHER_NAME[args.cipher]
     if args.workload == "c2":
         bits = args.bits or BITS_DEFAULT
         n = args.n or N_DEFAULT
-        return n * world, bits, "weak", f"configs[1]: MICKEY 2.0, {n} instances x {bits} bits per GPU per step"
+        return n * world, bits, "weak", f"configs[1]: {name}, {n} instances x {bits} bits per GPU per step"
+    if args.workload == "c4":
+        bits = args.bits or 4416
+        n = args.n or (1 << 19)
+        return n * world, bits, "weak", (f"configs[3]: {name} at the paper's launch shape (64 x 256 threads x 32 "
+                                         f"lanes = {n} instances) x {bits} clocks per GPU per step")
     bits = args.bits or (1 << 18)
     n_total = args.n or (1 << 25)
-    return n_total, bits, "strong", (f"configs[2]: MICKEY 2.0, {n_total} instances x {bits} bits in total, "
+    return n_total, bits, "strong", (f"configs[2]: {name}, {n_total} instances x {bits} bits in total, "
                                      f"split over {world} GPU(s)")
 
 
@@ -215,15 +233,15 @@ def run_reference(args, rank, world):
     cores = cpu_cores()
     n_s, bits_s = 64 * cores, 1 << 15
     for _ in range(args.warmup):
-        oracle_sample(n_s, bits_s, threads=cores)
+        oracle_sample(n_s, bits_s, threads=cores, cipher=args.cipher)
     tot_bits, tot_t = 0, 0.0
     for _ in range(args.steps):
-        r, dt = oracle_sample(n_s, bits_s, threads=cores)
+        r, dt = oracle_sample(n_s, bits_s, threads=cores, cipher=args.cipher)
         tot_bits += n_s * bits_s
         tot_t += dt
     v = tot_bits / tot_t / 1e12
     line = {
-        "impl": "reference", "metric": METRIC, "value": v, "unit": "Tb/s", "n_gpus": world,
+        "impl": "reference", "metric": metric(args), "value": v, "unit": "Tb/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": tot_t / args.steps * 1e3,
         "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "u32",
         "data": "synthetic (SplitMix64 keys/IVs, seed 0x5EED2020)",
@@ -247,20 +265,20 @@ def run_ours(args, rank, world, local_rank):
     dev = torch.device("cuda", local_rank)
     torch.cuda.set_device(dev)
     n_total, bits, scaling, desc = workload(args, world)
-    if args.workload == "c2":
+    if args.workload in ("c2", "c4"):
         first, n = shard.weak_range(rank, n_total // world)
     else:
         first, n = shard.strong_range(rank, world, n_total)
     stream = torch.cuda.Stream(dev)
 
-    keys_h, ivs_h = inputs.make_inputs("mickey2", n, first)
+    keys_h, ivs_h = inputs.make_inputs(args.cipher, n, first)
     keys_pin = torch.from_numpy(keys_h).pin_memory()
     ivs_pin = torch.from_numpy(ivs_h).pin_memory()
     keys_d = keys_pin.to(dev)
     ivs_d = ivs_pin.to(dev)
 
     with torch.cuda.stream(stream):
-        g = bsrng.Generator("mickey2", keys_d, ivs_d, first_instance=first, stream=stream)
+        g = bsrng.Generator(args.cipher, keys_d, ivs_d, first_instance=first, stream=stream)
     for k, v in (("sched", args.sched), ("seg_clocks", args.seg_clocks), ("ctas_per_sm", args.ctas_per_sm)):
         if v is not None:
             g.set_option(k, v)
@@ -327,7 +345,7 @@ def run_ours(args, rank, world, local_rank):
     nsm = torch.cuda.get_device_properties(dev).multi_processor_count
 
     def roofline(kern_ms_per_step, clocks):
-        lop3 = LOP3_PER_CLOCK * (n // 32) * bits       # algorithmic LOP3 per step, dominant kernel(s)
+        lop3 = LOP3_PER_CLOCK[args.cipher] * (n // 32) * bits  # algorithmic LOP3 per step, dominant kernel
         achieved = lop3 / (kern_ms_per_step * 1e-3) / 1e12
         peak = nsm * ALU_LANES_PER_SM_CLK * sm_max * 1e6 / 1e12
         out = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TLOP3/s", "frac": achieved / peak,
@@ -384,7 +402,7 @@ def run_ours(args, rank, world, local_rank):
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        cpu = cpu_baseline()
+        cpu = cpu_baseline(cipher=args.cipher)
     context = None
     if rank == 0 and world == 1 and not args.no_context:
         context = run_context(local_rank)
@@ -397,7 +415,7 @@ def run_ours(args, rank, world, local_rank):
             rf["traffic"] = tr.get("dram_bytes_per_launch")
             rf["traffic_note"] = tr.get("note")
         line = {
-            "metric": METRIC, "value": head["value"], "unit": "Tb/s", "n_gpus": world,
+            "metric": metric(args), "value": head["value"], "unit": "Tb/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": head["ms_per_step"],
             "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "u32",
             "data": "synthetic (SplitMix64 keys/IVs, seed 0x5EED2020)",

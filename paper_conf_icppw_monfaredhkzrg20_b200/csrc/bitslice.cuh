@@ -55,12 +55,29 @@ __device__ __forceinline__ void bt_stage8(uint32_t& a, uint32_t& b)
     b = nb;
 }
 
+// b << S and a >> S as integer multiplies (IMAD / IMAD.HI on the FMA pipe):
+// the keystream loop saturates the ALU pipe, the FMA pipe is idle.
+template <int S>
+__device__ __forceinline__ uint32_t shl_fma(uint32_t x)
+{
+    uint32_t d;
+    asm("mul.lo.u32 %0, %1, %2;" : "=r"(d) : "r"(x), "n"(1u << S));
+    return d;
+}
+template <int S>
+__device__ __forceinline__ uint32_t shr_fma(uint32_t x)
+{
+    uint32_t d;
+    asm("mul.hi.u32 %0, %1, %2;" : "=r"(d) : "r"(x), "n"(1u << (32 - S)));
+    return d;
+}
+
 template <int S, uint32_t M>
 __device__ __forceinline__ void bt_stage(uint32_t& a, uint32_t& b)
 {
     // element (r, c | S) <-> (r + S, c), c & S == 0; M = bits with c & S == 0
-    const uint32_t na = (a & M) | ((b << S) & ~M);
-    const uint32_t nb = ((a >> S) & M) | (b & ~M);
+    const uint32_t na = (a & M) | (shl_fma<S>(b) & ~M);
+    const uint32_t nb = (shr_fma<S>(a) & M) | (b & ~M);
     a = na;
     b = nb;
 }

@@ -20,6 +20,7 @@
 #include "keystream.cuh"
 #include "grain.cuh"
 #include "mickey2.cuh"
+#include "rowmajor_ws.cuh"
 
 namespace {
 
@@ -86,6 +87,7 @@ struct bsrng {
     // queue (measured: 78% vs 95% of the ALU roofline).
     int opt_ctas_per_sm = 1;
     int opt_unroll = KS_U_DEFAULT;
+    int opt_rm_ws = 1;  // ROW_MAJOR through the warp-specialised compute/writer kernel
 };
 
 namespace {
@@ -174,7 +176,19 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
     a.units = h->units;
     a.scratch = h->sched + 1 + h->units;
 
-    const size_t smem = LAYOUT == bsk::L_ROW_MAJOR ? size_t(KS_BLOCK / 32) * bsk::RM_WARP_WORDS * 4 : 0;
+    // ROW_MAJOR default: warp-specialised compute/writer kernel (rowmajor_ws.cuh),
+    // 8 warps per CTA of which 4 run the clock loop; always persistent.
+    const bool ws = LAYOUT == bsk::L_ROW_MAJOR && h->opt_rm_ws && h->opt_sched != 0;
+    int block = KS_BLOCK, compute_warps = KS_BLOCK / 32;
+    size_t smem = LAYOUT == bsk::L_ROW_MAJOR ? size_t(KS_BLOCK / 32) * bsk::RM_WARP_WORDS * 4 : 0;
+    if (ws) {
+        kern = &bsk::keystream_rm_ws_kernel<C, C::U_DEFAULT>;
+        if (h->opt_unroll == C::U_ALT0) kern = &bsk::keystream_rm_ws_kernel<C, C::U_ALT0>;
+        if (h->opt_unroll == C::U_ALT1) kern = &bsk::keystream_rm_ws_kernel<C, C::U_ALT1>;
+        block = bsk::ws::BLOCK;
+        compute_warps = bsk::ws::NCOMP;
+        smem = bsk::ws::SMEM_BYTES;
+    }
     if (smem > 48 * 1024) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
         if (e != cudaSuccess) return fail(BSRNG_ECUDA, "smem attribute: %s", cudaGetErrorString(e));
@@ -187,11 +201,11 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
         grid = unsigned((h->Gp + KS_BLOCK - 1) / KS_BLOCK);
     } else {
         int occ = h->opt_ctas_per_sm, occ_max = 1;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_max, kern, KS_BLOCK, smem) != cudaSuccess ||
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_max, kern, block, smem) != cudaSuccess ||
             occ_max < 1)
             occ_max = 1;
         if (occ <= 0 || occ > occ_max) occ = occ_max;
-        const uint64_t slots = uint64_t(h->num_sms) * occ * (KS_BLOCK / 32);  // resident warps
+        const uint64_t slots = uint64_t(h->num_sms) * occ * compute_warps;  // resident clock-loop warps
         uint64_t nseg = 1;
         if (h->opt_seg_clocks) {
             nseg = (bits + h->opt_seg_clocks - 1) / h->opt_seg_clocks;
@@ -211,7 +225,7 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
         a.ticket = h->sched;
         a.flags = h->sched + 1;
         const uint64_t items = h->units * nseg;
-        const uint64_t want_ctas = (items * 32 + KS_BLOCK - 1) / KS_BLOCK;
+        const uint64_t want_ctas = ws ? items : (items * 32 + KS_BLOCK - 1) / KS_BLOCK;
         grid = unsigned(std::min<uint64_t>(want_ctas, uint64_t(h->num_sms) * occ));
         cudaError_t e = cudaMemsetAsync(h->sched, 0, (1 + h->units) * sizeof(uint32_t), st);
         if (e != cudaSuccess) return fail(BSRNG_ECUDA, "memset(sched): %s", cudaGetErrorString(e));
@@ -227,7 +241,7 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
         cudaMemsetAsync(dbg, 0, 4 * sizeof(unsigned long long), st);
         a.dbg = dbg;
     }
-    kern<<<grid, KS_BLOCK, smem, st>>>(a);
+    kern<<<grid, block, smem, st>>>(a);
     int rc = check_launch("keystream");
     if (dbg) {
         unsigned long long c[4];
@@ -480,6 +494,9 @@ int bsrng_set_option(bsrng_t* h, const char* key, int64_t value)
                                              : (value == 2 || value == 4 || value == 8));
         if (!ok) return fail(BSRNG_EINVAL, "unroll must be %s", grain ? "8, 16 or 32" : "2, 4 or 8");
         h->opt_unroll = int(value);
+    } else if (!strcmp(key, "rm_ws")) {
+        if (value != 0 && value != 1) return fail(BSRNG_EINVAL, "rm_ws must be 0 or 1");
+        h->opt_rm_ws = int(value);
     } else if (!strcmp(key, "block")) {
         if (value != KS_BLOCK) return fail(BSRNG_EINVAL, "block=%lld not built (built: %d)", (long long)value, KS_BLOCK);
     } else {

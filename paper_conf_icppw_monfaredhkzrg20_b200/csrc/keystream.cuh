@@ -107,11 +107,15 @@ __device__ __forceinline__ void rowmajor_transpose(const uint32_t* zs, uint32_t*
 
 // Write slots [k_lo, k_hi] of every real row of this thread's group.
 //   row0: address of instance 32g's row; col: byte column of slot k_lo.
+// Full sectors go out as two 16 B stores (or four 8 B stores when rows are only
+// 8 B aligned, e.g. the paper's 4416-clock rows of 552 B); partial sectors at
+// item boundaries word by word.
 __device__ __forceinline__ void rowmajor_store(const uint32_t* os, uint8_t* row0, uint64_t row_bytes,
                                                uint32_t nvalid, uint32_t k_lo, uint32_t k_hi, uint64_t col)
 {
     uint8_t* p = row0 + col;
-    if (k_lo == 0 && k_hi == 7 && ((reinterpret_cast<uintptr_t>(p) | row_bytes) & 15) == 0) {
+    const uint64_t align = reinterpret_cast<uintptr_t>(p) | row_bytes;
+    if (k_lo == 0 && k_hi == 7 && (align & 15) == 0) {
 #pragma unroll 4
         for (uint32_t q = 0; q < nvalid; ++q) {
             const uint32_t* src = os + q * 8 * 32;
@@ -120,6 +124,16 @@ __device__ __forceinline__ void rowmajor_store(const uint32_t* os, uint8_t* row0
             uint4* d = reinterpret_cast<uint4*>(p + q * row_bytes);
             __stcs(d, v0);
             __stcs(d + 1, v1);
+        }
+    } else if (k_lo == 0 && k_hi == 7 && (align & 7) == 0) {
+#pragma unroll 4
+        for (uint32_t q = 0; q < nvalid; ++q) {
+            const uint32_t* src = os + q * 8 * 32;
+            uint2* d = reinterpret_cast<uint2*>(p + q * row_bytes);
+            __stcs(d, make_uint2(src[0], src[32]));
+            __stcs(d + 1, make_uint2(src[64], src[96]));
+            __stcs(d + 2, make_uint2(src[128], src[160]));
+            __stcs(d + 3, make_uint2(src[192], src[224]));
         }
     } else {
         for (uint32_t q = 0; q < nvalid; ++q)
