@@ -5,9 +5,11 @@ Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s
 product package ``paper_conf_icppw_monfaredhkzrg20_b200`` never imports it and
 shares no code with it.
 
-The arithmetic lives in plain C (``mickey2_ref.c``: bit-serial MICKEY 2.0,
-spec [5] cited at PAPER.md:870-871), compiled here into ``liboracle.so`` with
-gcc and called through ctypes.  This module only marshals arguments.
+The arithmetic lives in plain C -- ``mickey2_ref.c`` (bit-serial MICKEY 2.0,
+spec [5]), ``grain_ref.c`` (bit-serial Grain v1, spec [15],
+PAPER.md:898-899), ``aes_ref.c`` (byte-oriented AES-128 + CTR, FIPS-197 [35],
+PAPER.md:957-959) -- compiled here into ``liboracle.so`` with gcc and called
+through ctypes.  This module only marshals arguments.
 """
 from __future__ import annotations
 
@@ -19,7 +21,7 @@ from concurrent.futures import ThreadPoolExecutor
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-_SOURCES = ["mickey2_ref.c", "grain_ref.c"]
+_SOURCES = ["mickey2_ref.c", "grain_ref.c", "aes_ref.c"]
 _LIB_PATH = os.path.join(_HERE, "liboracle.so")
 _lib = None
 
@@ -57,6 +59,14 @@ def lib() -> ctypes.CDLL:
         L.ref_grain_state.restype = None
         L.ref_grain_clock.argtypes = [u8p, u8p, ctypes.c_int]
         L.ref_grain_clock.restype = ctypes.c_int
+        L.ref_aes128_encrypt_block.argtypes = [u8p, u8p, u8p]
+        L.ref_aes128_encrypt_block.restype = None
+        L.ref_aes128_expand_key.argtypes = [u8p, u8p]
+        L.ref_aes128_expand_key.restype = None
+        L.ref_aes_sbox.argtypes = [ctypes.c_uint8]
+        L.ref_aes_sbox.restype = ctypes.c_uint8
+        L.ref_aes128_ctr_keystream.argtypes = [u8p, u8p, ctypes.c_uint64, ctypes.c_uint64, u8p]
+        L.ref_aes128_ctr_keystream.restype = None
         _lib = L
     return _lib
 
@@ -187,3 +197,55 @@ def grain_keystream_batch(keys: np.ndarray, ivs: np.ndarray, nbits: int, threads
         with ThreadPoolExecutor(max_workers=threads) as ex:
             list(ex.map(one, range(n)))
     return out[:, :nbytes]
+
+
+# --------------------------------------------------------------- AES-128-CTR
+def aes128_encrypt_block(key: bytes, block: bytes) -> bytes:
+    k = _buf(key, 16)
+    b = _buf(block, 16)
+    out = np.zeros(16, dtype=np.uint8)
+    lib().ref_aes128_encrypt_block(_p(k), _p(b), _p(out))
+    return out.tobytes()
+
+
+def aes128_expand_key(key: bytes) -> bytes:
+    k = _buf(key, 16)
+    w = np.zeros(176, dtype=np.uint8)
+    lib().ref_aes128_expand_key(_p(k), _p(w))
+    return w.tobytes()
+
+
+def aes_sbox() -> np.ndarray:
+    return np.array([lib().ref_aes_sbox(x) for x in range(256)], dtype=np.uint8)
+
+
+def aes128_ctr_keystream(key: bytes, ctr: bytes, nblocks: int, first_block: int = 0) -> bytes:
+    k = _buf(key, 16)
+    c = _buf(ctr, 16)
+    out = np.zeros(max(16 * nblocks, 1), dtype=np.uint8)
+    lib().ref_aes128_ctr_keystream(_p(k), _p(c), first_block, nblocks, _p(out))
+    return out[: 16 * nblocks].tobytes()
+
+
+def aes128_ctr_keystream_batch(key: bytes, ctrs: np.ndarray, nbits: int, first_block: int = 0,
+                               threads: int | None = None) -> np.ndarray:
+    """Row-major AES-CTR keystreams of n counter streams under one key:
+    uint8[n, nbits/8]; nbits must be a multiple of 128."""
+    assert nbits % 128 == 0
+    k = _buf(key, 16)
+    ctrs = np.ascontiguousarray(ctrs, dtype=np.uint8)
+    n = ctrs.shape[0]
+    out = np.zeros((n, max(nbits // 8, 1)), dtype=np.uint8)
+    L = lib()
+
+    def one(i):
+        L.ref_aes128_ctr_keystream(_p(k), _p(ctrs[i]), first_block, nbits // 128, _p(out[i]))
+
+    threads = threads or os.cpu_count() or 1
+    if threads == 1 or n == 1:
+        for i in range(n):
+            one(i)
+    else:
+        with ThreadPoolExecutor(max_workers=threads) as ex:
+            list(ex.map(one, range(n)))
+    return out[:, : nbits // 8]

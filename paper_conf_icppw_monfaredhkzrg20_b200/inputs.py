@@ -21,6 +21,11 @@ MICKEY 2.0     LE(x0) || LE(x1)[0:2]  (10 B)    LE(x2) || LE(x3)[0:2]  (10 B)
 Grain v1       LE(x0) || LE(x1)[0:2]  (10 B)    LE(x2)                 (8 B)
 AES-128-CTR    LE(x0) || LE(x1)       (16 B)    LE(x2) || LE(x3)       (16 B)
 =============  ==============================  ==============================
+
+AES-128-CTR runs every instance under ONE key ("different
+counter values ... with a unique key"): the handle key is global instance 0's
+key row, ``aes_key(seed)``, whatever shard is being generated; each instance's
+IV row is its initial 128-bit big-endian counter block.
 """
 from __future__ import annotations
 
@@ -67,3 +72,9 @@ def make_inputs(cipher: str, n: int, first_instance: int = 0, seed: int = DEFAUL
     keys = np.concatenate([xb[:, 0, :], xb[:, 1, :]], axis=1)[:, :kb]
     ivs = np.concatenate([xb[:, 2, :], xb[:, 3, :]], axis=1)[:, :vb]
     return np.ascontiguousarray(keys), np.ascontiguousarray(ivs)
+
+
+def aes_key(seed: int = DEFAULT_SEED) -> np.ndarray:
+    """The single AES-128 key of a seeded workload: global instance 0's key row."""
+    keys, _ = make_inputs("aes128ctr", 1, 0, seed)
+    return keys[0].copy()
