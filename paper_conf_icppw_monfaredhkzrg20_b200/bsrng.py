@@ -23,7 +23,7 @@ OK, EINVAL, ENOMEM, ECUDA, ERANGE, EUNSUPPORTED = 0, -1, -2, -3, -4, -5
 
 CIPHERS = {"mickey2": MICKEY2, "grain": GRAIN_V1, "aes128ctr": AES128_CTR}
 LAYOUTS = {"row_major": ROW_MAJOR, "sliced": SLICED, "checksum": CHECKSUM}
-NSTATE = {MICKEY2: 200, GRAIN_V1: 160}
+NSTATE = {MICKEY2: 200, GRAIN_V1: 160, AES128_CTR: 128}
 DEFAULT_IV_BITS = {MICKEY2: 80, GRAIN_V1: 64, AES128_CTR: 128}
 
 SYMBOLS = [
@@ -138,7 +138,9 @@ class Generator:
         self.iv_bits = DEFAULT_IV_BITS.get(self.cipher, 0) if iv_bits is None else int(iv_bits)
         kp, kdev = _ptr(keys)
         vp, vdev = _ptr(ivs)
-        n = int(keys.shape[0]) if hasattr(keys, "shape") else 0
+        # AES-128-CTR: ONE key for all instances, n = number of counter blocks
+        rows = ivs if self.cipher == AES128_CTR else keys
+        n = int(rows.shape[0]) if hasattr(rows, "shape") else 0
         self._keep = (keys, ivs)  # host arrays must outlive the async copy
         flags = INPUT_DEVICE if kdev else INPUT_HOST
         if ivs is not None and vdev != kdev:
@@ -154,6 +156,8 @@ class Generator:
     @classmethod
     def from_seed(cls, cipher, n, first_instance=0, seed=_inputs.DEFAULT_SEED, **kw):
         keys, ivs = _inputs.make_inputs(cipher, n, first_instance, seed)
+        if cipher in ("aes128ctr", AES128_CTR):
+            keys = _inputs.aes_key(seed)
         return cls(cipher, keys, ivs, first_instance=first_instance, **kw)
 
     # -- properties -------------------------------------------------------
