@@ -16,7 +16,7 @@ ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 def _sources():
     out = [os.path.join(ROOT, "include", "bsrng.h")]
     for f in sorted(os.listdir(CSRC)):
-        if f.endswith((".cu", ".cuh", ".h")):
+        if f.endswith((".cu", ".cuh", ".h", ".inc")):
             out.append(os.path.join(CSRC, f))
     return out
 

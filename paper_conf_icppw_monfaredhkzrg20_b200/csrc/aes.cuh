@@ -19,8 +19,8 @@
 //   counter: x = base + T (128-bit big-endian add of the warp-uniform block
 //            index T to the sliced initial counters, ripple carry), fused with
 //            round-0 AddRoundKey                                  ~256 LOP3
-//   SubBytes: 16 x the Boyar-Peralta depth-16 S-box circuit (113 gates:
-//            32 AND, 81 XOR/XNOR; verified against the S-box table)
+//   SubBytes: 16 x the Boyar-Peralta depth-16 S-box circuit as 84 LOP3s
+//            (tools/lut3_map.py; 113 two-input gates originally)
 //   ShiftRows: register renaming; MixColumns + AddRoundKey: XOR trees.
 // AES-CTR has no state carried between blocks: work items of one instance in
 // different time segments are independent (no segment flags).
@@ -39,44 +39,23 @@ struct RoundKeys {
     uint32_t m[11][128];
 };
 
-// Boyar-Peralta S-box circuit on one byte: u[0] = MSB ... u[7] = LSB (in place).
+// AES S-box on one byte held MSB-first in 8 slice words (in place): the
+// Boyar-Peralta depth-16 circuit (113 two-input gates) mapped onto 84
+// three-input LOP3s by tools/lut3_map.py (cut enumeration + area recovery),
+// verified there against the FIPS-197 S-box on all 256 inputs.
 __device__ __forceinline__ void sbox(uint32_t& U0, uint32_t& U1, uint32_t& U2, uint32_t& U3, uint32_t& U4,
                                      uint32_t& U5, uint32_t& U6, uint32_t& U7)
 {
-    const uint32_t T1 = U0 ^ U3, T2 = U0 ^ U5, T3 = U0 ^ U6, T4 = U3 ^ U5, T5 = U4 ^ U6;
-    const uint32_t T6 = T1 ^ T5, T7 = U1 ^ U2, T8 = U7 ^ T6, T9 = U7 ^ T7, T10 = T6 ^ T7;
-    const uint32_t T11 = U1 ^ U5, T12 = U2 ^ U5, T13 = T3 ^ T4, T14 = T6 ^ T11, T15 = T5 ^ T11;
-    const uint32_t T16 = T5 ^ T12, T17 = T9 ^ T16, T18 = U3 ^ U7, T19 = T7 ^ T18, T20 = T1 ^ T19;
-    const uint32_t T21 = U6 ^ U7, T22 = T7 ^ T21, T23 = T2 ^ T22, T24 = T2 ^ T10, T25 = T20 ^ T17;
-    const uint32_t T26 = T3 ^ T16, T27 = T1 ^ T12;
-    const uint32_t D = U7;
-    const uint32_t M1 = T13 & T6, M2 = T23 & T8, M3 = T14 ^ M1, M4 = T19 & D, M5 = M4 ^ M1;
-    const uint32_t M6 = T3 & T16, M7 = T22 & T9, M8 = T26 ^ M6, M9 = T20 & T17, M10 = M9 ^ M6;
-    const uint32_t M11 = T1 & T15, M12 = T4 & T27, M13 = M12 ^ M11, M14 = T2 & T10, M15 = M14 ^ M11;
-    const uint32_t M16 = M3 ^ M2, M17 = M5 ^ T24, M18 = M8 ^ M7, M19 = M10 ^ M15, M20 = M16 ^ M13;
-    const uint32_t M21 = M17 ^ M15, M22 = M18 ^ M13, M23 = M19 ^ T25, M24 = M22 ^ M23, M25 = M22 & M20;
-    const uint32_t M26 = M21 ^ M25, M27 = M20 ^ M21, M28 = M23 ^ M25, M29 = M28 & M27, M30 = M26 & M24;
-    const uint32_t M31 = M20 & M23, M32 = M27 & M31, M33 = M27 ^ M25, M34 = M21 & M22, M35 = M24 & M34;
-    const uint32_t M36 = M24 ^ M25, M37 = M21 ^ M29, M38 = M32 ^ M33, M39 = M23 ^ M30, M40 = M35 ^ M36;
-    const uint32_t M41 = M38 ^ M40, M42 = M37 ^ M39, M43 = M37 ^ M38, M44 = M39 ^ M40, M45 = M42 ^ M41;
-    const uint32_t M46 = M44 & T6, M47 = M40 & T8, M48 = M39 & D, M49 = M43 & T16, M50 = M38 & T9;
-    const uint32_t M51 = M37 & T17, M52 = M42 & T15, M53 = M45 & T27, M54 = M41 & T10, M55 = M44 & T13;
-    const uint32_t M56 = M40 & T23, M57 = M39 & T19, M58 = M43 & T3, M59 = M38 & T22, M60 = M37 & T20;
-    const uint32_t M61 = M42 & T1, M62 = M45 & T4, M63 = M41 & T2;
-    const uint32_t L0 = M61 ^ M62, L1 = M50 ^ M56, L2 = M46 ^ M48, L3 = M47 ^ M55, L4 = M54 ^ M58;
-    const uint32_t L5 = M49 ^ M61, L6 = M62 ^ L5, L7 = M46 ^ L3, L8 = M51 ^ M59, L9 = M52 ^ M53;
-    const uint32_t L10 = M53 ^ L4, L11 = M60 ^ L2, L12 = M48 ^ M51, L13 = M50 ^ L0, L14 = M52 ^ M61;
-    const uint32_t L15 = M55 ^ L1, L16 = M56 ^ L0, L17 = M57 ^ L1, L18 = M58 ^ L8, L19 = M63 ^ L4;
-    const uint32_t L20 = L0 ^ L1, L21 = L1 ^ L7, L22 = L3 ^ L12, L23 = L18 ^ L2, L24 = L15 ^ L9;
-    const uint32_t L25 = L6 ^ L10, L26 = L7 ^ L9, L27 = L8 ^ L10, L28 = L11 ^ L14, L29 = L11 ^ L17;
-    U0 = L6 ^ L24;
-    U1 = ~(L16 ^ L26);
-    U2 = ~(L19 ^ L28);
-    U3 = L6 ^ L21;
-    U4 = L20 ^ L22;
-    U5 = L25 ^ L29;
-    U6 = ~(L13 ^ L27);
-    U7 = ~(L6 ^ L23);
+    uint32_t S0, S1, S2, S3, S4, S5, S6, S7;
+#include "aes_sbox_lop3.inc"
+    U0 = S0;
+    U1 = S1;
+    U2 = S2;
+    U3 = S3;
+    U4 = S4;
+    U5 = S5;
+    U6 = S6;
+    U7 = S7;
 }
 
 __device__ __forceinline__ void sub_bytes(uint32_t (&s)[128])
@@ -102,43 +81,42 @@ __device__ __forceinline__ void shift_rows(uint32_t (&s)[128])
     for (int i = 0; i < 128; ++i) s[i] = t[i];
 }
 
-// xtime on one byte held MSB-first in v[0..7]: result bit i (significance)
-// is v<<1 with 0x1b folded in where the old MSB was set.
-__device__ __forceinline__ void xtime(const uint32_t (&v)[8], uint32_t (&o)[8])
-{
-    // significance k <-> index 7-k
-    o[7] = v[0];          // bit0 = old bit7
-    o[6] = v[7] ^ v[0];   // bit1 = old bit0 ^ bit7
-    o[5] = v[6];          // bit2 = old bit1
-    o[4] = v[5] ^ v[0];   // bit3 = old bit2 ^ bit7
-    o[3] = v[4] ^ v[0];   // bit4 = old bit3 ^ bit7
-    o[2] = v[3];          // bit5 = old bit4
-    o[1] = v[2];          // bit6 = old bit5
-    o[0] = v[1];          // bit7 = old bit6
-}
-
-// MixColumns (FIPS-197 5.1.3) + AddRoundKey with round-key row `k` (masks).
+// MixColumns (FIPS-197 5.1.3) + AddRoundKey with round-key row `k` (masks),
+// two LOP3 per output bit.  With u_i = a_i ^ a_{i+1} (indices mod 4):
+//   out_i = 2a_i ^ 3a_{i+1} ^ a_{i+2} ^ a_{i+3} ^ k = a_{i+1} ^ u_{i+2} ^ xtime(u_i) ^ k
+// and xtime(u) = (u << 1) ^ (u_7 ? 0x1b : 0) adds u_7 at significance 0, 1, 3, 4.
+// Byte words are MSB-first: significance s lives at index 7 - s.
 __device__ __forceinline__ void mix_columns_ark(uint32_t (&s)[128], const uint32_t* k)
 {
+    constexpr uint32_t X3 = 0xF0u ^ 0xCCu ^ 0xAAu;  // a ^ b ^ c
+    constexpr uint32_t X2 = 0xF0u ^ 0xCCu;          // a ^ b
 #pragma unroll
     for (int c = 0; c < 4; ++c) {
-        uint32_t a[4][8];
+        uint32_t u[4][8];
 #pragma unroll
         for (int i = 0; i < 4; ++i)
 #pragma unroll
-            for (int b = 0; b < 8; ++b) a[i][b] = s[8 * (4 * c + i) + b];
-        uint32_t t[8];
-#pragma unroll
-        for (int b = 0; b < 8; ++b) t[b] = a[0][b] ^ a[1][b] ^ a[2][b] ^ a[3][b];
+            for (int b = 0; b < 8; ++b) u[i][b] = s[8 * (4 * c + i) + b] ^ s[8 * (4 * c + ((i + 1) & 3)) + b];
+        uint32_t o[4][8];
 #pragma unroll
         for (int i = 0; i < 4; ++i) {
-            uint32_t u[8], x[8];
+            const uint32_t* a1 = &s[8 * (4 * c + ((i + 1) & 3))];
+            const uint32_t* kk = &k[8 * (4 * c + i)];
 #pragma unroll
-            for (int b = 0; b < 8; ++b) u[b] = a[i][b] ^ a[(i + 1) & 3][b];
-            xtime(u, x);
-#pragma unroll
-            for (int b = 0; b < 8; ++b) s[8 * (4 * c + i) + b] = a[i][b] ^ t[b] ^ x[b] ^ k[8 * (4 * c + i) + b];
+            for (int sig = 0; sig < 8; ++sig) {
+                const int b = 7 - sig;
+                const uint32_t xt = sig == 0 ? u[i][0] : u[i][b + 1];  // (u << 1) at significance sig
+                const uint32_t t = lop3<X3>(a1[b], u[(i + 2) & 3][b], xt);
+                if (sig == 1 || sig == 3 || sig == 4)
+                    o[i][b] = lop3<X3>(t, u[i][0], kk[b]);  // + u_7 (index 0) from the 0x1b reduction
+                else
+                    o[i][b] = lop3<X2>(t, kk[b], 0u);
+            }
         }
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+#pragma unroll
+            for (int b = 0; b < 8; ++b) s[8 * (4 * c + i) + b] = o[i][b];
     }
 }
 
@@ -240,7 +218,7 @@ __global__ void aes_key_expand_kernel(const uint8_t* __restrict__ key, uint32_t*
 //              (two encryptions fill a sector) and written as 16 B stores.
 // ---------------------------------------------------------------------------
 template <int LAYOUT>
-__global__ void __launch_bounds__(128, 1) aes_ctr_kernel(const KsArgs a, const __grid_constant__ aes::RoundKeys rk)
+__global__ void __launch_bounds__(128, 2) aes_ctr_kernel(const KsArgs a, const __grid_constant__ aes::RoundKeys rk)
 {
     constexpr int NW = 4;
     extern __shared__ uint32_t aes_smem[];  // base counters [128][128 threads] (+ ROW_MAJOR sector buffers)

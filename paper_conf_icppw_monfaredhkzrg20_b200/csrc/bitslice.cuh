@@ -10,6 +10,17 @@
 
 namespace bsk {
 
+// One explicit 3-input logic op: d = LUT(a, b, c), LUT bit 4a+2b+c
+// (truth tables written as F(0xF0, 0xCC, 0xAA)).  Inline PTX keeps the
+// compiler from re-associating hand-chosen LOP3 trees.
+template <uint32_t LUT>
+__device__ __forceinline__ uint32_t lop3(uint32_t a, uint32_t b, uint32_t c)
+{
+    uint32_t d;
+    asm("lop3.b32 %0, %1, %2, %3, %4;" : "=r"(d) : "r"(a), "r"(b), "r"(c), "n"(LUT));
+    return d;
+}
+
 // ---------------------------------------------------------------------------
 // Key/IV slicing (SURVEY step a-1; "32x80 bits of IV for each
 // thread").  One warp per group g: lane j holds instance 32g+j's byte string;

@@ -91,7 +91,7 @@ struct bsrng {
     // enough ILP to keep the ALU pipe busy, and with two warps per SMSP the
     // issue arbiter starves one of them, which stalls the time-segmented work
     // queue (measured: 78% vs 95% of the ALU roofline).
-    int opt_ctas_per_sm = 1;
+    int opt_ctas_per_sm = 0;  // 0 = default: 1 (stream ciphers), 2 (AES-CTR)
     int opt_unroll = KS_U_DEFAULT;
     int opt_rm_ws = 1;  // ROW_MAJOR through the warp-specialised compute/writer kernel
 };
@@ -227,7 +227,8 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_max, kern, block, smem) != cudaSuccess ||
             occ_max < 1)
             occ_max = 1;
-        if (occ <= 0 || occ > occ_max) occ = occ_max;
+        if (occ <= 0) occ = 1;
+        if (occ > occ_max) occ = occ_max;
         const uint64_t slots = uint64_t(h->num_sms) * occ * compute_warps;  // resident clock-loop warps
         uint64_t nseg = 1;
         if (h->opt_seg_clocks) {
@@ -304,7 +305,17 @@ int launch_aes(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
     const size_t smem = size_t(128) * 128 * 4 + (LAYOUT == bsk::L_ROW_MAJOR ? size_t(4) * bsk::OS_WORDS * 4 : 0);
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
     if (e != cudaSuccess) return fail(BSRNG_ECUDA, "smem attribute: %s", cudaGetErrorString(e));
-    const uint64_t slots = uint64_t(h->num_sms) * 4;
+    // Two warps per SMSP (two CTAs per SM) when shared memory allows: the
+    // second warp hides the round-key constant loads (short-scoreboard stalls)
+    // and AES work items never wait on each other, so the issue arbiter's
+    // favouritism cannot stall the queue.  ROW_MAJOR's sector buffers limit
+    // it to one CTA per SM.
+    int occ = h->opt_ctas_per_sm > 0 ? h->opt_ctas_per_sm : 2;
+    int occ_max = 1;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_max, kern, 128, smem) != cudaSuccess || occ_max < 1)
+        occ_max = 1;
+    occ = std::min(occ, occ_max);
+    const uint64_t slots = uint64_t(h->num_sms) * occ * 4;
     const uint64_t quantum = bits >= 256 ? 256 : 128;
     uint64_t nseg = h->opt_seg_clocks ? (bits + h->opt_seg_clocks - 1) / h->opt_seg_clocks
                                       : (32 * slots + h->units - 1) / h->units;
@@ -320,7 +331,7 @@ int launch_aes(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
     }
     if (e != cudaSuccess) return fail(BSRNG_ECUDA, "memset: %s", cudaGetErrorString(e));
     const uint64_t items = h->units * a.nseg;
-    const unsigned grid = unsigned(std::min<uint64_t>((items + 3) / 4, uint64_t(h->num_sms)));
+    const unsigned grid = unsigned(std::min<uint64_t>((items + 3) / 4, uint64_t(h->num_sms) * occ));
     kern<<<grid, 128, smem, st>>>(a, h->rk);
     return check_launch("aes_ctr");
 }

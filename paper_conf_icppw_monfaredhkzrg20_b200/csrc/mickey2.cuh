@@ -36,22 +36,12 @@ __host__ __device__ constexpr bool fb1(int i) { return pick(0x4C8CB877u, 0x4911B
 
 constexpr int NSTATE = 200;
 
-// a ^ (b & c) as one explicit LOP3.  Written as inline PTX because, given the
-// C expression, the compiler folds CONTROL_BIT_R = s34 ^ r67 into every AND
+// a ^ (b & c) as one explicit LOP3 (bsk::lop3, bitslice.cuh).  Given the C
+// expression, the compiler folds CONTROL_BIT_R = s34 ^ r67 into every AND
 // (r_i & (s34 ^ r67) is one 3-input LOP3) and then needs a second LOP3 for the
 // XOR with r_{i-1}: 2 ops per bit instead of 1 (+50 ops per clock).
 constexpr uint32_t LUT_A_XOR_BC = 0xF0u ^ (0xCCu & 0xAAu);  // 0x78
-template <uint32_t LUT>
-__device__ __forceinline__ uint32_t lop3(uint32_t a, uint32_t b, uint32_t c)
-{
-    uint32_t d;
-    asm("lop3.b32 %0, %1, %2, %3, %4;" : "=r"(d) : "r"(a), "r"(b), "r"(c), "n"(LUT));
-    return d;
-}
 
-// s'_I = s^_I ^ (feedback term of category (FB0_I, FB1_I)).  s^_I is one LOP3
-// whose truth table folds COMP0_I / COMP1_I in at compile time (explicit PTX:
-// left to itself ptxas keeps some s_i complemented and pays NOTs for them).
 template <int I>
 __device__ __forceinline__ uint32_t s_next(const uint32_t (&s)[100], uint32_t fb_s, uint32_t fb_s0, uint32_t fb_s1)
 {
