@@ -35,8 +35,10 @@ sys.path.insert(0, ROOT)
 N_DEFAULT = 1 << 22
 BITS_DEFAULT = 1 << 20
 # algorithmic LOP3 per clock per 32-instance group
-LOP3_PER_CLOCK = {"mickey2": 327, "grain": 39}
-CIPHER_NAME = {"mickey2": "MICKEY 2.0", "grain": "Grain v1"}
+# (AES-128-CTR: 17280 LOP3 per 32-block encryption = 4096 bits per group,
+#  i.e. 135 per keystream bit position per group)
+LOP3_PER_CLOCK = {"mickey2": 327, "grain": 39, "aes128ctr": 135}
+CIPHER_NAME = {"mickey2": "MICKEY 2.0", "grain": "Grain v1", "aes128ctr": "AES-128-CTR"}
 ALU_LANES_PER_SM_CLK = 64      # 4 SMSP x 16 lanes (alu pipe rt = 2 cycles/warp-instr)
 METRIC = "MICKEY 2.0 keystream Tb/s (1 and 8 B200); fraction of LOP3/HBM roofline"
 
@@ -56,7 +58,7 @@ def parse():
                    help="c2 = BASELINE configs[1] per GPU (weak scaling); "
                         "c3 = configs[2]: 2^25 instances x 2^18 bits = 1 TiB total, split across GPUs (strong); "
                         "c4 = configs[3]: the paper's launch shape, 2^19 instances x 4416 clocks per GPU")
-    p.add_argument("--cipher", default="mickey2", choices=["mickey2", "grain"])
+    p.add_argument("--cipher", default="mickey2", choices=["mickey2", "grain", "aes128ctr"])
     p.add_argument("--n", type=int, default=None, help="instances per GPU (c2) / in total (c3)")
     p.add_argument("--bits", type=int, default=None, help="keystream bits per instance per step")
     p.add_argument("--no-context", action="store_true", help="skip the ALU-peak / cuRAND microbenchmarks")
@@ -167,6 +169,8 @@ def oracle_sample(n_inst, bits, first=0, threads=None, cipher="mickey2"):
     t = time.perf_counter()
     if cipher == "grain":
         oracle.grain_keystream_batch(keys, ivs, bits, threads=threads)
+    elif cipher == "aes128ctr":
+        oracle.aes128_ctr_keystream_batch(bytes(inputs.aes_key()), ivs, bits // 128 * 128, threads=threads)
     else:
         oracle.mickey2_keystream_batch(keys, ivs, 80, bits, threads=threads)
     dt = time.perf_counter() - t
@@ -216,7 +220,7 @@ def workload(args, world):
         n = args.n or N_DEFAULT
         return n * world, bits, "weak", f"configs[1]: {name}, {n} instances x {bits} bits per GPU per step"
     if args.workload == "c4":
-        bits = args.bits or 4416
+        bits = args.bits or (4480 if args.cipher == "aes128ctr" else 4416)
         n = args.n or (1 << 19)
         return n * world, bits, "weak", (f"configs[3]: {name} at the paper's launch shape (64 x 256 threads x 32 "
                                          f"lanes = {n} instances) x {bits} clocks per GPU per step")
@@ -272,6 +276,8 @@ def run_ours(args, rank, world, local_rank):
     stream = torch.cuda.Stream(dev)
 
     keys_h, ivs_h = inputs.make_inputs(args.cipher, n, first)
+    if args.cipher == "aes128ctr":
+        keys_h = inputs.aes_key()  # one key for every instance
     keys_pin = torch.from_numpy(keys_h).pin_memory()
     ivs_pin = torch.from_numpy(ivs_h).pin_memory()
     keys_d = keys_pin.to(dev)
