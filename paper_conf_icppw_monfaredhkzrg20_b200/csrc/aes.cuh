@@ -149,6 +149,53 @@ __device__ __forceinline__ void counter_block(uint32_t (&s)[128], const uint32_t
 // ten of them (300 KB) do not -- ncu showed `no_instruction` as the dominant
 // stall with the rounds unrolled.  Round keys are read with a warp-uniform
 // runtime index from the kernel-parameter constant bank.
+// Block-lane layout (ROW_MAJOR kernel below): the 32 lanes of a thread are 32
+// CONSECUTIVE blocks V + j of ONE instance.  V is the 128-bit big-endian block
+// value of lane 0 (V[0] most significant).  With c = V mod 32, H = V >> 5:
+//   significance 0..4 of block j = bits of (c + j) mod 32 -> the lane patterns
+//     0xAAAAAAAA, 0xCCCCCCCC, ... rotated right by c;
+//   significance 5..127 = bits of H, or of H + 1 in the lanes j >= 32 - c that
+//     carried out of the low five bits.
+// Round key 0 is folded in: the K0 bits >= 5 are XORed into H and H + 1 before
+// the per-bit masks are extracted.
+__device__ __forceinline__ uint32_t bit_mask(uint32_t w, int q)
+{
+    return uint32_t(int32_t(w << (31 - q)) >> 31);  // 0 or ~0
+}
+
+__device__ __forceinline__ void counter_block_lanes(uint32_t (&s)[128], const uint32_t (&V)[4], const RoundKeys& rk,
+                                                    const uint32_t (&K0hi)[4])
+{
+    const uint32_t c = V[3] & 31u;
+    const uint32_t carry = c ? (0xFFFFFFFFu << (32 - c)) : 0u;
+    uint32_t H[4], H1[4];
+    H[3] = (V[3] >> 5) | (V[2] << 27);
+    H[2] = (V[2] >> 5) | (V[1] << 27);
+    H[1] = (V[1] >> 5) | (V[0] << 27);
+    H[0] = V[0] >> 5;
+    uint32_t cy = 1u;
+#pragma unroll
+    for (int w = 3; w >= 0; --w) {
+        H1[w] = H[w] + cy;
+        cy = (cy && H1[w] == 0u) ? 1u : 0u;
+    }
+#pragma unroll
+    for (int w = 0; w < 4; ++w) {
+        H[w] ^= K0hi[w];
+        H1[w] ^= K0hi[w];
+    }
+    constexpr uint32_t P0[5] = {0xAAAAAAAAu, 0xCCCCCCCCu, 0xF0F0F0F0u, 0xFF00FF00u, 0xFFFF0000u};
+#pragma unroll
+    for (int p = 0; p < 5; ++p) s[127 - p] = __funnelshift_r(P0[p], P0[p], c) ^ rk.m[0][127 - p];
+#pragma unroll
+    for (int p = 5; p < 128; ++p) {
+        const int q = p - 5;
+        const uint32_t m0 = bit_mask(H[3 - (q >> 5)], q & 31);
+        const uint32_t m1 = bit_mask(H1[3 - (q >> 5)], q & 31);
+        s[127 - p] = (carry & m1) | (~carry & m0);
+    }
+}
+
 __device__ __forceinline__ void encrypt(uint32_t (&s)[128], const RoundKeys& rk)
 {
 #pragma unroll 1
@@ -317,6 +364,115 @@ __global__ void __launch_bounds__(128, 2) aes_ctr_kernel(const KsArgs a, const _
                     for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(0xFFFFFFFFu, v, off);
                     if (lane == 0) atomicAdd(static_cast<unsigned long long*>(a.out), (unsigned long long)v);
                 }
+            }
+        }
+        next_item(a, slot);
+    }
+}
+
+// ---------------------------------------------------------------------------
+// ROW_MAJOR in the block-lane layout: thread = ONE instance, lane j = block
+// V + j.  After the rounds, transposing the four 32x32 tiles in registers
+// leaves block j's 16 bytes in s[j], s[32+j], s[64+j], s[96+j]: one 16 B
+// store per block, 512 contiguous bytes of the instance's row per
+// encryption -- whole sectors with no shared-memory staging.  Used when a call
+// has >= 32 blocks per instance (otherwise most lanes would be wasted).
+// Work items: (time segment of whole 4096-bit encryptions, 32-instance warp);
+// `a.units` counts warps here, `a.aux` = row-major initial counters (n x 16 B).
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(128, 2) aes_ctr_rowmajor_lanes_kernel(const KsArgs a,
+                                                                         const __grid_constant__ aes::RoundKeys rk)
+{
+    __shared__ uint32_t s_item[4];
+    volatile uint32_t* slot = s_item + (threadIdx.x >> 5);
+    next_item(a, slot);
+    const uint64_t total = a.units * a.nseg;
+    uint32_t K0hi[4];  // bits >= 5 of round key 0 as a 123-bit value (H's alignment)
+    {
+        uint32_t K[4] = {0, 0, 0, 0};
+#pragma unroll
+        for (int b = 0; b < 128; ++b) K[b >> 5] |= (rk.m[0][b] & 1u) << (31 - (b & 31));
+        K0hi[3] = (K[3] >> 5) | (K[2] << 27);
+        K0hi[2] = (K[2] >> 5) | (K[1] << 27);
+        K0hi[1] = (K[1] >> 5) | (K[0] << 27);
+        K0hi[0] = K[0] >> 5;
+    }
+    for (;;) {
+        const uint64_t item = *slot;
+        if (item >= total) break;
+        const uint32_t lane = threadIdx.x & 31u;
+        const uint64_t seg = item / a.units;
+        const uint64_t w = item - seg * a.units;
+        const uint64_t inst = w * 32u + lane;
+        const bool real = inst < a.n;
+        const uint64_t bit_begin = seg * a.seg_clocks;
+        const uint64_t left = a.nclocks - bit_begin;
+        const uint64_t nblocks = (left < a.seg_clocks ? left : a.seg_clocks) >> 7;
+        // V = ctr_inst + first block index of this item (128-bit big-endian)
+        uint32_t V[4] = {0, 0, 0, 0};
+        if (real) {
+            const uint8_t* cb = static_cast<const uint8_t*>(a.aux) + inst * 16;
+#pragma unroll
+            for (int k = 0; k < 4; ++k)
+                V[k] = (uint32_t(cb[4 * k]) << 24) | (uint32_t(cb[4 * k + 1]) << 16) | (uint32_t(cb[4 * k + 2]) << 8) |
+                       uint32_t(cb[4 * k + 3]);
+        }
+        {
+            const uint64_t T = (a.t0 + bit_begin) >> 7;
+            uint64_t lo = (uint64_t(V[2]) << 32) | V[3];
+            uint64_t hi = (uint64_t(V[0]) << 32) | V[1];
+            const uint64_t nlo = lo + T;
+            hi += (nlo < lo) ? 1u : 0u;
+            lo = nlo;
+            V[0] = uint32_t(hi >> 32);
+            V[1] = uint32_t(hi);
+            V[2] = uint32_t(lo >> 32);
+            V[3] = uint32_t(lo);
+        }
+        uint8_t* row = static_cast<uint8_t*>(a.out) + (real ? inst : 0) * a.row_bytes + (bit_begin >> 3);
+#pragma unroll 1
+        for (uint64_t blk = 0; blk < nblocks; blk += 32) {
+            uint32_t s[128];
+            aes::counter_block_lanes(s, V, rk, K0hi);
+            aes::encrypt(s, rk);
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                uint32_t x0[16], x1[16];
+#pragma unroll
+                for (int q = 0; q < 16; ++q) {
+                    const uint32_t lo = s[32 * k + (q ^ 7)], hi = s[32 * k + ((q + 16) ^ 7)];
+                    x0[q] = __byte_perm(lo, hi, 0x5410);
+                    x1[q] = __byte_perm(lo, hi, 0x7632);
+                }
+                bt_transpose16(x0);
+                bt_transpose16(x1);
+#pragma unroll
+                for (int q = 0; q < 16; ++q) {
+                    s[32 * k + q] = x0[q];
+                    s[32 * k + 16 + q] = x1[q];
+                }
+            }
+            const uint64_t nb = nblocks - blk < 32 ? nblocks - blk : 32;
+            if (real) {
+                uint4* dst = reinterpret_cast<uint4*>(row + blk * 16);
+                if (nb == 32) {
+#pragma unroll
+                    for (int j = 0; j < 32; ++j) __stcs(dst + j, make_uint4(s[j], s[32 + j], s[64 + j], s[96 + j]));
+                } else {
+#pragma unroll
+                    for (int j = 0; j < 32; ++j)
+                        if (uint64_t(j) < nb) __stcs(dst + j, make_uint4(s[j], s[32 + j], s[64 + j], s[96 + j]));
+                }
+            }
+            // V += 32
+            const uint32_t v3 = V[3] + 32u;
+            uint32_t cy = v3 < V[3] ? 1u : 0u;
+            V[3] = v3;
+#pragma unroll
+            for (int k = 2; k >= 0; --k) {
+                const uint32_t t = V[k] + cy;
+                cy = (cy && t == 0u) ? 1u : 0u;
+                V[k] = t;
             }
         }
         next_item(a, slot);

@@ -336,6 +336,44 @@ int launch_aes(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
     return check_launch("aes_ctr");
 }
 
+// AES ROW_MAJOR with >= 32 blocks per instance: block-lane kernel (aes.cuh).
+int launch_aes_rowmajor_lanes(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
+{
+    auto kern = &bsk::aes_ctr_rowmajor_lanes_kernel;
+    bsk::KsArgs a{};
+    a.n = h->n;
+    a.G = h->G;
+    a.Gp = h->Gp;
+    a.nclocks = bits;
+    a.t0 = h->bits_done;
+    a.out = out;
+    a.row_bytes = bits / 8;
+    a.units = h->G;  // one warp = 32 instances
+    a.aux = h->raw + h->key_rows * h->key_bytes;
+    a.persistent = 1;
+    a.ticket = h->sched;
+    a.flags = h->sched + 1;
+    int occ = h->opt_ctas_per_sm > 0 ? h->opt_ctas_per_sm : 2;
+    int occ_max = 1;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_max, kern, 128, 0) != cudaSuccess || occ_max < 1)
+        occ_max = 1;
+    occ = std::min(occ, occ_max);
+    const uint64_t slots = uint64_t(h->num_sms) * occ * 4;
+    const uint64_t quantum = 4096;  // one 32-block encryption per instance
+    uint64_t nseg = h->opt_seg_clocks ? (bits + h->opt_seg_clocks - 1) / h->opt_seg_clocks
+                                      : (32 * slots + a.units - 1) / a.units;
+    nseg = std::max<uint64_t>(1, std::min<uint64_t>(nseg, (bits + quantum - 1) / quantum));
+    const uint64_t seg = ((bits + nseg - 1) / nseg + quantum - 1) / quantum * quantum;
+    a.nseg = (bits + seg - 1) / seg;
+    a.seg_clocks = seg;
+    cudaError_t e = cudaMemsetAsync(h->sched, 0, sizeof(uint32_t), st);
+    if (e != cudaSuccess) return fail(BSRNG_ECUDA, "memset: %s", cudaGetErrorString(e));
+    const uint64_t items = a.units * a.nseg;
+    const unsigned grid = unsigned(std::min<uint64_t>((items + 3) / 4, uint64_t(h->num_sms) * occ));
+    kern<<<grid, 128, 0, st>>>(a, h->rk);
+    return check_launch("aes_ctr_rowmajor_lanes");
+}
+
 template <class C>
 int dispatch_layout(bsrng_t* h, void* out, uint64_t bits, bsrng_layout layout, cudaStream_t st)
 {
@@ -489,7 +527,8 @@ int bsrng_generate(bsrng_t* h, void* out, uint64_t bits, bsrng_layout layout, vo
     case BSRNG_MICKEY2: rc = dispatch_layout<bsk::Mickey2>(h, out, bits, layout, st); break;
     case BSRNG_GRAIN_V1: rc = dispatch_layout<bsk::Grain>(h, out, bits, layout, st); break;
     case BSRNG_AES128_CTR:
-        rc = layout == BSRNG_ROW_MAJOR ? launch_aes<bsk::L_ROW_MAJOR>(h, out, bits, st)
+        rc = layout == BSRNG_ROW_MAJOR ? (bits >= 4096 && h->opt_rm_ws ? launch_aes_rowmajor_lanes(h, out, bits, st)
+                                                                       : launch_aes<bsk::L_ROW_MAJOR>(h, out, bits, st))
              : layout == BSRNG_SLICED  ? launch_aes<bsk::L_SLICED>(h, out, bits, st)
                                        : launch_aes<bsk::L_CHECKSUM>(h, out, bits, st);
         break;

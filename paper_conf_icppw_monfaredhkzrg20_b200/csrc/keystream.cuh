@@ -51,6 +51,7 @@ struct KsArgs {
     uint32_t* ticket;     // persistent mode: [1], zeroed before launch
     uint32_t* flags;      // persistent mode: [units], zeroed before launch
     uint32_t* scratch;    // [32] sink for padding-group SLICED stores
+    const void* aux;      // cipher-specific input (AES block-lane ROW_MAJOR: counters)
     unsigned long long* dbg;  // optional scheduler counters (BSRNG_DEBUG), or null
     int persistent;
 };

@@ -90,3 +90,25 @@ def test_large_sampled():
     idx = np.unique(np.concatenate([np.random.default_rng(3).integers(0, n, 128), [0, 31, 32, n - 1]]))
     want = oracle.aes128_ctr_keystream_batch(bytes(key), ctrs[idx], bits)
     assert np.array_equal(rows[idx], want)
+
+
+@pytest.mark.parametrize("bits,seg", [(4096, 0), (4096 * 3 + 1024, 0), (4096 * 5, 4096), (8192, 8192)])
+def test_rowmajor_block_lanes(bits, seg):
+    """ROW_MAJOR calls with >= 32 blocks per instance take the block-lane
+    kernel (lanes = consecutive blocks of one instance); partial last
+    encryptions, segments and a preceding call (block offset) included."""
+    n = 32 * 5 + 3
+    _, ctrs = inputs.make_inputs("aes128ctr", n)
+    ctrs = ctrs.copy()
+    ctrs[7] = np.frombuffer(bytes([0xFF] * 15 + [0xF0]), np.uint8)   # 128-bit wrap inside a 32-block tile
+    ctrs[8, 8:] = 0xFF
+    ctrs[8, 15] = 0xE1                                               # carry out of the low 64 bits
+    key = inputs.aes_key()
+    g = bsrng.Generator("aes128ctr", key, ctrs)
+    if seg:
+        g.set_option("seg_clocks", seg)
+    pre = g.generate_host(384, "checksum")  # 3 blocks consumed first
+    got = g.generate_host(bits, "row_major")
+    want = oracle.aes128_ctr_keystream_batch(bytes(key), ctrs, bits, first_block=3)
+    assert np.array_equal(got, want)
+    assert int(pre[0]) == checksum(to_sliced(oracle.aes128_ctr_keystream_batch(bytes(key), ctrs, 384)))
