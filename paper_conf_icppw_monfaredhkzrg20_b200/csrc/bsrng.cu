@@ -87,11 +87,8 @@ struct bsrng {
     // options
     int opt_sched = 1;
     uint64_t opt_seg_clocks = 0;
-    // One resident CTA (4 warps) per SM = one warp per SMSP: a single warp has
-    // enough ILP to keep the ALU pipe busy, and with two warps per SMSP the
-    // issue arbiter starves one of them, which stalls the time-segmented work
-    // queue (measured: 78% vs 95% of the ALU roofline).
-    int opt_ctas_per_sm = 0;  // 0 = default: 1 (stream ciphers), 2 (AES-CTR)
+    // Resident CTAs per SM; 0 = auto (launch_keystream / launch_aes).
+    int opt_ctas_per_sm = 0;
     int opt_unroll = KS_U_DEFAULT;
     int opt_rm_ws = 1;  // ROW_MAJOR through the warp-specialised compute/writer kernel
 };
@@ -227,13 +224,24 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_max, kern, block, smem) != cudaSuccess ||
             occ_max < 1)
             occ_max = 1;
-        if (occ <= 0) occ = 1;
+        // Auto policy (opt_ctas_per_sm == 0).  Many more warp-units than warp
+        // slots: two warps per SMSP, one item per unit (no time segments, so no
+        // warp ever waits on another; a warp left alone at the end runs at
+        // nearly full rate).  Otherwise: one warp per SMSP and time segments,
+        // so the tail is one segment long (with two warps per SMSP the issue
+        // arbiter starves one of them and segment hand-offs stall).
+        bool whole_units = false;
+        if (occ <= 0) {
+            const uint64_t slots2 = uint64_t(h->num_sms) * 2 * compute_warps;
+            whole_units = !ws && occ_max >= 2 && h->units >= 3 * slots2;
+            occ = whole_units ? 2 : 1;
+        }
         if (occ > occ_max) occ = occ_max;
         const uint64_t slots = uint64_t(h->num_sms) * occ * compute_warps;  // resident clock-loop warps
         uint64_t nseg = 1;
         if (h->opt_seg_clocks) {
             nseg = (bits + h->opt_seg_clocks - 1) / h->opt_seg_clocks;
-        } else if (h->units > slots) {
+        } else if (!whole_units && h->units > slots) {
             // >= ~32 items per resident warp so the tail is <~3% of the call,
             // but segments no shorter than 256 clocks (state carry stays <1%)
             nseg = std::max<uint64_t>(1, (32 * slots + h->units - 1) / h->units);

@@ -9,8 +9,8 @@
 //
 // Both registers shift by one position per clock (Fibonacci form), so the
 // shift is pure register renaming; only the three new words (f, g, z) cost
-// logic: ~39 LOP3 per clock per 32 keystream bits, 8x cheaper
-// than MICKEY 2.0.  The renaming closes every 80 clocks; with U clocks per loop
+// logic: 37 LOP3 per clock per 32 keystream bits (f 3, g 25, h + z 9; SURVEY
+// App. D estimated 39), ~9x cheaper than MICKEY 2.0.  The renaming closes every 80 clocks; with U clocks per loop
 // iteration ptxas restores the register map at the back edge with moves
 // (160/U per clock, issued on the otherwise idle FMA pipe).
 #pragma once
@@ -23,50 +23,70 @@ namespace grain {
 
 constexpr int NSTATE = 160;  // s_0..s_79, b_0..b_79
 
-// h(x0..x4) = x1+x4+x0x3+x2x3+x3x4+x0x1x2+x0x2x3+x0x2x4+x1x2x4+x2x3x4
-//           = [x1 + x4 + x3(x0 + x4)] + x2 [x3 + x0x1 + x0x3 + x0x4 + x1x4 + x3x4]
-__device__ __forceinline__ uint32_t h_filter(uint32_t x0, uint32_t x1, uint32_t x2, uint32_t x3, uint32_t x4)
+// LOP3 truth tables (a = 0xF0, b = 0xCC, c = 0xAA)
+constexpr uint32_t XOR3 = 0x96u, XOR2 = 0x3Cu, AND3 = 0x80u, AND2 = 0xC0u;
+constexpr uint32_t XAND = 0x78u;  // a ^ (b & c)
+constexpr uint32_t MUX = 0xCAu;   // a ? b : c
+
+// Output z = b1+b2+b4+b10+b31+b43+b56 + h(s3, s25, s46, s64, b63), with
+//   h = x1 + x4 + x0x3 + x2x3 + x3x4 + x0x1x2 + x0x2x3 + x0x2x4 + x1x2x4 + x2x3x4
+//     = x1 + (x3 ? x0 : x4) + x2 * B,
+//   B = x0 ? (x1|x4) + x3x4 : x3 + x1x4 + x3x4          (x0 = s3, x1 = s25,
+// x2 = s46, x3 = s64, x4 = b63; verified exhaustively in DESIGN.md's note).
+// `extra` is XORed in (the checksum accumulator, or 0): 9 LOP3 (+1 with extra).
+template <bool EXTRA>
+__device__ __forceinline__ uint32_t output(const uint32_t (&s)[80], const uint32_t (&b)[80], uint32_t extra = 0u)
 {
-    const uint32_t a = x1 ^ x4 ^ (x3 & (x0 ^ x4));
-    const uint32_t b = x3 ^ (x0 & x1) ^ (x0 & x3) ^ (x0 & x4) ^ (x1 & x4) ^ (x3 & x4);
-    return a ^ (x2 & b);
+    const uint32_t x0 = s[3], x1 = s[25], x2 = s[46], x3 = s[64], x4 = b[63];
+    const uint32_t m = lop3<MUX>(x3, x0, x4);
+    const uint32_t B0 = lop3<0xE4u>(x1, x3, x4);  // x3 ^ x1x4 ^ x3x4
+    const uint32_t B1 = lop3<0x72u>(x1, x3, x4);  // (x1 | x4) ^ x3x4
+    const uint32_t B = lop3<MUX>(x0, B1, B0);
+    const uint32_t w1 = lop3<XOR3>(b[1], b[2], b[4]);
+    const uint32_t w2 = lop3<XOR3>(b[10], b[31], b[43]);
+    const uint32_t w3 = lop3<XOR3>(b[56], x1, m);
+    uint32_t w = lop3<XOR3>(w1, w2, w3);
+    if (EXTRA) w = lop3<XOR2>(w, extra, 0u);
+    return lop3<XAND>(w, x2, B);
 }
 
-// z = b1+b2+b4+b10+b31+b43+b56 + h(s3, s25, s46, s64, b63)
-__device__ __forceinline__ uint32_t output(const uint32_t (&s)[80], const uint32_t (&b)[80])
-{
-    return b[1] ^ b[2] ^ b[4] ^ b[10] ^ b[31] ^ b[43] ^ b[56] ^ h_filter(s[3], s[25], s[46], s[64], b[63]);
-}
-
-// f: s_80 = s62+s51+s38+s23+s13+s0
+// f: s_80 = s62+s51+s38+s23+s13+s0  (3 LOP3)
 __device__ __forceinline__ uint32_t f_lfsr(const uint32_t (&s)[80])
 {
-    return s[62] ^ s[51] ^ s[38] ^ s[23] ^ s[13] ^ s[0];
+    return lop3<XOR3>(lop3<XOR3>(s[62], s[51], s[38]), lop3<XOR3>(s[23], s[13], s[0]), 0u);
 }
 
 // g: b_80 = s0 + b62+b60+b52+b45+b37+b33+b28+b21+b14+b9+b0 + b63b60 + b37b33 + b15b9
 //         + b60b52b45 + b33b28b21 + b63b45b28b9 + b60b52b37b33 + b63b60b21b15
 //         + b63b60b52b45b37 + b33b28b21b15b9 + b52b45b37b33b28b21
-// with the shared products p60_63, p33_37, p9_15, p45_52, p21_28.
+// as a balanced LOP3 tree: 25 ops, depth 5 (the linear terms are grouped
+// with single AND-products into a ^ (b & c) gates).
 __device__ __forceinline__ uint32_t g_nfsr(uint32_t s0, const uint32_t (&b)[80])
 {
-    const uint32_t p60_63 = b[63] & b[60];
-    const uint32_t p33_37 = b[37] & b[33];
-    const uint32_t p9_15 = b[15] & b[9];
-    const uint32_t p45_52 = b[52] & b[45];
-    const uint32_t p21_28 = b[28] & b[21];
-    const uint32_t p21_28_33 = p21_28 & b[33];
-    uint32_t v = s0 ^ b[62] ^ b[60] ^ b[52] ^ b[45] ^ b[37] ^ b[33] ^ b[28] ^ b[21] ^ b[14] ^ b[9] ^ b[0];
-    v ^= p60_63 ^ p33_37 ^ p9_15;
-    v ^= b[60] & p45_52;
-    v ^= p21_28_33;
-    v ^= (b[63] & b[45]) & (b[28] & b[9]);
-    v ^= b[60] & b[52] & p33_37;
-    v ^= p60_63 & b[21] & b[15];
-    v ^= p60_63 & p45_52 & b[37];
-    v ^= p21_28_33 & p9_15;
-    v ^= p45_52 & p33_37 & p21_28;
-    return v;
+    const uint32_t t1 = lop3<XOR3>(s0, b[62], b[60]);
+    const uint32_t t2 = lop3<XOR3>(b[52], b[45], b[37]);
+    const uint32_t t3 = lop3<XOR3>(b[33], b[28], b[21]);
+    const uint32_t t4 = lop3<XOR3>(b[14], b[9], b[0]);
+    const uint32_t q45 = lop3<AND2>(b[52], b[45], 0u);
+    const uint32_t q21 = lop3<AND2>(b[28], b[21], 0u);
+    const uint32_t p1 = lop3<AND2>(b[63], b[60], 0u);
+    const uint32_t p2 = lop3<AND2>(b[37], b[33], 0u);
+    const uint32_t p3 = lop3<AND2>(b[15], b[9], 0u);
+    const uint32_t a1 = lop3<XAND>(t2, b[60], q45);        // + b60b52b45
+    const uint32_t p5 = lop3<AND2>(b[33], q21, 0u);        // b33b28b21
+    const uint32_t m1 = lop3<AND2>(b[63], b[45], 0u);
+    const uint32_t m2 = lop3<AND2>(b[28], b[9], 0u);
+    const uint32_t a2 = lop3<XAND>(t3, m1, m2);            // + b63b45b28b9
+    const uint32_t p7 = lop3<AND3>(b[60], b[52], p2);      // b60b52b37b33
+    const uint32_t p8 = lop3<AND3>(p1, b[21], b[15]);      // b63b60b21b15
+    const uint32_t p9 = lop3<AND3>(p1, q45, b[37]);        // b63b60b52b45b37
+    const uint32_t a3 = lop3<XAND>(t4, p5, p3);            // + b33b28b21b15b9
+    const uint32_t p11 = lop3<AND3>(q45, p2, q21);         // b52b45b37b33b28b21
+    const uint32_t u1 = lop3<XOR3>(t1, a1, a2);
+    const uint32_t u2 = lop3<XOR3>(a3, p1, p2);
+    const uint32_t u3 = lop3<XOR3>(p3, p5, p7);
+    const uint32_t u4 = lop3<XOR3>(p8, p9, p11);
+    return lop3<XOR3>(lop3<XOR3>(u1, u2, u3), u4, 0u);
 }
 
 // One clock.  INIT = the initialisation mode: z is added to both feedbacks.
@@ -76,9 +96,9 @@ __device__ __forceinline__ void clock(uint32_t (&s)[80], uint32_t (&b)[80])
     uint32_t fs = f_lfsr(s);
     uint32_t fb = g_nfsr(s[0], b);
     if (INIT) {
-        const uint32_t z = output(s, b);
-        fs ^= z;
-        fb ^= z;
+        const uint32_t z = output<false>(s, b);
+        fs = lop3<XOR2>(fs, z, 0u);
+        fb = lop3<XOR2>(fb, z, 0u);
     }
 #pragma unroll
     for (int i = 0; i < 79; ++i) {
@@ -117,7 +137,9 @@ struct Grain {
 #pragma unroll
         for (int i = 0; i < 80; ++i) __stcg(p + uint64_t(80 + i) * Gp, b[i]);
     }
-    __device__ __forceinline__ uint32_t z() const { return grain::output(s, b); }
+    __device__ __forceinline__ uint32_t z() const { return grain::output<false>(s, b); }
+    // checksum accumulation fused into the output XOR tree
+    __device__ __forceinline__ uint32_t z_acc(uint32_t acc) const { return grain::output<true>(s, b, acc); }
     __device__ __forceinline__ void clock() { grain::clock<false>(s, b); }
 };
 

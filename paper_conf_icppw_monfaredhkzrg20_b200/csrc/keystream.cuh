@@ -106,6 +106,22 @@ __device__ __forceinline__ void rowmajor_transpose(const uint32_t* zs, uint32_t*
     }
 }
 
+// The same from 32 z words held in registers (cipher loops unrolled 32x).
+template <bool MSB_FIRST>
+__device__ __forceinline__ void rowmajor_transpose_regs(const uint32_t (&z)[32], uint32_t* os, uint32_t k)
+{
+    constexpr int X = MSB_FIRST ? 7 : 0;
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+        uint32_t x[16];
+#pragma unroll
+        for (int q = 0; q < 16; ++q) x[q] = __byte_perm(z[q ^ X], z[(q + 16) ^ X], h == 0 ? 0x5410 : 0x7632);
+        bt_transpose16(x);
+#pragma unroll
+        for (int q = 0; q < 16; ++q) os[((16 * h + q) * 8 + k) * 32] = x[q];
+    }
+}
+
 // Write slots [k_lo, k_hi] of every real row of this thread's group.
 //   row0: address of instance 32g's row; col: byte column of slot k_lo.
 // Full sectors go out as two 16 B stores (or four 8 B stores when rows are only
@@ -216,7 +232,7 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
             for (uint32_t it = nclk / U; it != 0; --it) {
 #pragma unroll
                 for (int u = 0; u < U; ++u) {
-                    acc ^= c.z();
+                    acc = c.z_acc(acc);
                     c.clock();
                 }
             }
@@ -245,17 +261,29 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
             const uint32_t nblk = nclk >> 5;
 #pragma unroll 1
             for (uint32_t blk = 0; blk < nblk; ++blk) {
-#pragma unroll 1
-                for (uint32_t k = 0; k < 32; k += U) {
-#pragma unroll
-                    for (int u = 0; u < U; ++u) {
-                        zs[(k + u) * 32] = c.z();
-                        c.clock();
-                    }
-                }
                 const uint64_t B = b0 + blk;
                 const uint32_t k = uint32_t(B & 7);
-                rowmajor_transpose<C::MSB_FIRST>(zs, zs + ZS_WORDS, k);
+                if constexpr (U == 32) {
+                    // one 32-clock block per iteration: keep the z words in
+                    // registers and transpose them there (no z staging in smem)
+                    uint32_t zr[32];
+#pragma unroll
+                    for (int u = 0; u < 32; ++u) {
+                        zr[u] = c.z();
+                        c.clock();
+                    }
+                    rowmajor_transpose_regs<C::MSB_FIRST>(zr, zs + ZS_WORDS, k);
+                } else {
+#pragma unroll 1
+                    for (uint32_t kk = 0; kk < 32; kk += U) {
+#pragma unroll
+                        for (int u = 0; u < U; ++u) {
+                            zs[(kk + u) * 32] = c.z();
+                            c.clock();
+                        }
+                    }
+                    rowmajor_transpose<C::MSB_FIRST>(zs, zs + ZS_WORDS, k);
+                }
                 if (k == 7 || blk + 1 == nblk) {
                     const uint32_t k_lo = k - (blk < k ? blk : k);
                     rowmajor_store(zs + ZS_WORDS, s_row0[threadIdx.x], a.row_bytes, s_nvalid[threadIdx.x], k_lo,

@@ -139,6 +139,7 @@ struct Mickey2 {
     }
     // keystream bit z = r0 ^ s0, taken before the clock (spec [5])
     __device__ __forceinline__ uint32_t z() const { return r[0] ^ s[0]; }
+    __device__ __forceinline__ uint32_t z_acc(uint32_t acc) const { return acc ^ r[0] ^ s[0]; }
     __device__ __forceinline__ void clock() { m2::clock_kg<false>(r, s, 0u); }
 };
 

@@ -24,12 +24,18 @@ def main():
     p.add_argument("--reps", type=int, default=3)
     p.add_argument("--sched", type=int, default=None)
     p.add_argument("--seg-clocks", type=int, default=None)
+    p.add_argument("--rm-ws", type=int, default=None)
+    p.add_argument("--unroll", type=int, default=None)
     a = p.parse_args()
     g = bsrng.Generator.from_seed(a.cipher, a.n)
     if a.sched is not None:
         g.set_option("sched", a.sched)
     if a.seg_clocks is not None:
         g.set_option("seg_clocks", a.seg_clocks)
+    if a.rm_ws is not None:
+        g.set_option("rm_ws", a.rm_ws)
+    if a.unroll is not None:
+        g.set_option("unroll", a.unroll)
     out = torch.empty(max(g.out_bytes(a.bits, a.layout), 16), dtype=torch.uint8, device="cuda")
     for _ in range(a.reps):
         g.generate(out, a.bits, a.layout)
