@@ -34,10 +34,17 @@ sys.path.insert(0, ROOT)
 
 N_DEFAULT = 1 << 22
 BITS_DEFAULT = 1 << 20
-# algorithmic LOP3 per clock per 32-instance group
-# (AES-128-CTR: 17280 LOP3 per 32-block encryption = 4096 bits per group,
-#  i.e. 135 per keystream bit position per group)
-LOP3_PER_CLOCK = {"mickey2": 327, "grain": 39, "aes128ctr": 135}
+# Algorithmic LOP3 per keystream bit position per 32-instance group (DESIGN.md
+# sec. 5): MICKEY 2.0 327 per clock (output op included);
+# Grain v1 37 per clock (f 3 + g 25 + h/z 9) + 1 to fold into the checksum;
+# AES-128-CTR 17280 per 32-block encryption (4096 bit positions) + 64 for the
+# checksum XOR tree.
+def lop3_per_bit(cipher, mode):
+    if cipher == "mickey2":
+        return 327.0
+    if cipher == "grain":
+        return 38.0 if mode == "consume" else 37.0
+    return (17280.0 + (64.0 if mode == "consume" else 0.0)) / 128.0
 CIPHER_NAME = {"mickey2": "MICKEY 2.0", "grain": "Grain v1", "aes128ctr": "AES-128-CTR"}
 ALU_LANES_PER_SM_CLK = 64      # 4 SMSP x 16 lanes (alu pipe rt = 2 cycles/warp-instr)
 METRIC = "MICKEY 2.0 keystream Tb/s (1 and 8 B200); fraction of LOP3/HBM roofline"
@@ -350,8 +357,8 @@ def run_ours(args, rank, world, local_rank):
     sm_max = float(peaks.get("sm_max_mhz", 1965.0))
     nsm = torch.cuda.get_device_properties(dev).multi_processor_count
 
-    def roofline(kern_ms_per_step, clocks):
-        lop3 = LOP3_PER_CLOCK[args.cipher] * (n // 32) * bits  # algorithmic LOP3 per step, dominant kernel
+    def roofline(kern_ms_per_step, clocks, mode):
+        lop3 = lop3_per_bit(args.cipher, mode) * (n // 32) * bits  # algorithmic LOP3 per step, dominant kernel
         achieved = lop3 / (kern_ms_per_step * 1e-3) / 1e12
         peak = nsm * ALU_LANES_PER_SM_CLK * sm_max * 1e6 / 1e12
         out = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TLOP3/s", "frac": achieved / peak,
@@ -371,7 +378,7 @@ def run_ours(args, rank, world, local_rank):
         tbps = n_total * bits / (ms * 1e-3) / 1e12
         res = {"value": tbps, "ms_per_step": ms, "kernel_ms_per_step": kms,
                "kernel_tbps_per_gpu": n * bits / (kms * 1e-3) / 1e12,
-               "gpu_launches": launches, "roofline": roofline(kms, clocks)}
+               "gpu_launches": launches, "roofline": roofline(kms, clocks, mode)}
         if mode == "materialise":
             out_bytes = n * bits / 8
             res["hbm_write_gbs_per_gpu"] = out_bytes / (kms * 1e-3) / 1e9
