@@ -61,10 +61,11 @@ def parse():
     p.add_argument("--steps", type=int, default=3)
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    p.add_argument("--workload", default="c2", choices=["c2", "c3", "c4"],
+    p.add_argument("--workload", default="c2", choices=["c2", "c3", "c4", "rekey"],
                    help="c2 = BASELINE configs[1] per GPU (weak scaling); "
                         "c3 = configs[2]: 2^25 instances x 2^18 bits = 1 TiB total, split across GPUs (strong); "
-                        "c4 = configs[3]: the paper's launch shape, 2^19 instances x 4416 clocks per GPU")
+                        "c4 = configs[3]: the paper's launch shape, 2^19 instances x 4416 clocks per GPU; "
+                        "rekey = SURVEY NEXT-3: 2^22 short streams x 2^10 bits, key/IV setup dominates")
     p.add_argument("--cipher", default="mickey2", choices=["mickey2", "grain", "aes128ctr"])
     p.add_argument("--n", type=int, default=None, help="instances per GPU (c2) / in total (c3)")
     p.add_argument("--bits", type=int, default=None, help="keystream bits per instance per step")
@@ -226,6 +227,11 @@ def workload(args, world):
         bits = args.bits or BITS_DEFAULT
         n = args.n or N_DEFAULT
         return n * world, bits, "weak", f"configs[1]: {name}, {n} instances x {bits} bits per GPU per step"
+    if args.workload == "rekey":
+        bits = args.bits or 1024
+        n = args.n or N_DEFAULT
+        return n * world, bits, "weak", (f"NEXT-3 rekey: {name}, {n} fresh keys/IVs x {bits} bits per GPU per step "
+                                         f"(slicing + initialisation clocks + keystream)")
     if args.workload == "c4":
         bits = args.bits or (4480 if args.cipher == "aes128ctr" else 4416)
         n = args.n or (1 << 19)
@@ -276,7 +282,7 @@ def run_ours(args, rank, world, local_rank):
     dev = torch.device("cuda", local_rank)
     torch.cuda.set_device(dev)
     n_total, bits, scaling, desc = workload(args, world)
-    if args.workload in ("c2", "c4"):
+    if args.workload in ("c2", "c4", "rekey"):
         first, n = shard.weak_range(rank, n_total // world)
     else:
         first, n = shard.strong_range(rank, world, n_total)
@@ -303,6 +309,8 @@ def run_ours(args, rank, world, local_rank):
             dist.barrier()
 
     def step_consume(ev=None):
+        if ev:
+            ev[2].record(stream)
         g.rekey(keys_d, ivs_d, stream=stream)
         if ev:
             ev[0].record(stream)
@@ -317,6 +325,8 @@ def run_ours(args, rank, world, local_rank):
         nonlocal rm_buf
         if rm_buf is None:
             rm_buf = torch.empty(g.out_bytes(chunk, "row_major"), dtype=torch.uint8, device=dev)
+        if ev:
+            ev[2].record(stream)
         g.rekey(keys_d, ivs_d, stream=stream)
         if ev:
             ev[0].record(stream)
@@ -329,7 +339,7 @@ def run_ours(args, rank, world, local_rank):
         for _ in range(warmup):
             step_fn()
         torch.cuda.synchronize(dev)
-        step_ms, kern_ms = [], []
+        step_ms, kern_ms, rekey_ms = [], [], []
         l0 = bsrng.launch_count()
         if sampler:
             sampler.start()
@@ -339,23 +349,38 @@ def run_ours(args, rank, world, local_rank):
             barrier()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             k0, k1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            r0 = torch.cuda.Event(enable_timing=True)
             e0.record(stream)
-            step_fn((k0, k1))
+            step_fn((k0, k1, r0))
             e1.record(stream)
             torch.cuda.synchronize(dev)
             barrier()
             step_ms.append(e0.elapsed_time(e1))
             kern_ms.append(k0.elapsed_time(k1))
+            rekey_ms.append(r0.elapsed_time(k0))
         clocks = sampler.stop() if sampler else None
         launches = bsrng.launch_count() - l0
-        t = torch.tensor([sum(step_ms), sum(kern_ms)], dtype=torch.float64, device=dev)
+        t = torch.tensor([sum(step_ms), sum(kern_ms), sum(rekey_ms)], dtype=torch.float64, device=dev)
         if world > 1:
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        timed.rekey_ms = float(t[2]) / steps
         return float(t[0]) / steps, float(t[1]) / steps, launches, clocks
 
     peaks = measured_peaks()
     sm_max = float(peaks.get("sm_max_mhz", 1965.0))
     nsm = torch.cuda.get_device_properties(dev).multi_processor_count
+
+    def init_roofline(rk_ms):
+        """a-1 + a-2 (bsrng_rekey) against the same ALU peak: initialisation
+        clocks x ops per clock (MICKEY 260 x 328, Grain 160 x 39; AES-CTR has
+        no initialisation clocks, only slicing + a one-thread key expansion)."""
+        ops = {"mickey2": 260 * 328.0, "grain": 160 * 39.0}.get(args.cipher)
+        if not ops or rk_ms <= 0:
+            return None
+        achieved = ops * (n // 32) / (rk_ms * 1e-3) / 1e12
+        peak = nsm * ALU_LANES_PER_SM_CLK * sm_max * 1e6 / 1e12
+        return {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TLOP3/s", "frac": achieved / peak,
+                "note": "rekey = slice kernels + preclock kernel (+ H2D for e2e)"}
 
     def roofline(kern_ms_per_step, clocks, mode):
         lop3 = lop3_per_bit(args.cipher, mode) * (n // 32) * bits  # algorithmic LOP3 per step, dominant kernel
@@ -376,7 +401,10 @@ def run_ours(args, rank, world, local_rank):
         sampler = ClockSampler(local_rank) if (rank == 0 and mode == args.mode) else None
         ms, kms, launches, clocks = timed(fn, args.steps, args.warmup, sampler)
         tbps = n_total * bits / (ms * 1e-3) / 1e12
+        rk_ms = timed.rekey_ms
         res = {"value": tbps, "ms_per_step": ms, "kernel_ms_per_step": kms,
+               "rekey_ms_per_step": rk_ms, "keys_per_s": n_total / (rk_ms * 1e-3) if rk_ms > 0 else None,
+               "preclock_roofline": init_roofline(rk_ms),
                "kernel_tbps_per_gpu": n * bits / (kms * 1e-3) / 1e12,
                "gpu_launches": launches, "roofline": roofline(kms, clocks, mode)}
         if mode == "materialise":
@@ -399,6 +427,8 @@ def run_ours(args, rank, world, local_rank):
         cs_host = torch.zeros(1, dtype=torch.int64).pin_memory()
 
         def step_e2e(ev=None):
+            if ev:
+                ev[2].record(stream)
             g.rekey(keys_pin.numpy(), ivs_pin.numpy(), stream=stream)
             if ev:
                 ev[0].record(stream)

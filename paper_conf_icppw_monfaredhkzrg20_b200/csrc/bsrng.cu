@@ -121,12 +121,12 @@ int run_init(bsrng_t* h, cudaStream_t st)
     uint32_t* iv_s = h->sliced + kbits * h->Gp;
     const uint8_t* raw_k = h->raw;
     const uint8_t* raw_iv = h->raw + h->key_rows * h->key_bytes;
-    const unsigned sblocks = unsigned((h->Gp * 32 + 255) / 256);
+    const unsigned sblocks = unsigned((h->Gp + 31) / 32);  // 32 groups per 1024-thread block
     switch (h->cipher) {
     case BSRNG_MICKEY2: {
-        bsk::slice_bits_kernel<10, 80, true><<<sblocks, 256, 0, st>>>(raw_k, h->n, key_s, h->Gp);
+        bsk::slice_bits_kernel<10, 80, true><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_k, h->n, key_s, h->Gp);
         if (int rc = check_launch("slice(key)")) return rc;
-        bsk::slice_bits_kernel<10, 80, true><<<sblocks, 256, 0, st>>>(raw_iv, h->n, iv_s, h->Gp);
+        bsk::slice_bits_kernel<10, 80, true><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_iv, h->n, iv_s, h->Gp);
         if (int rc = check_launch("slice(iv)")) return rc;
         const unsigned pblocks = unsigned((h->Gp + 127) / 128);
         bsk::m2_preclock_kernel<<<pblocks, 128, 0, st>>>(iv_s, key_s, int(h->iv_bits), h->state, h->Gp);
@@ -136,9 +136,9 @@ int run_init(bsrng_t* h, cudaStream_t st)
     }
     case BSRNG_GRAIN_V1: {
         // spec [15]: key and IV bits are taken LSB-first from their bytes
-        bsk::slice_bits_kernel<10, 80, false><<<sblocks, 256, 0, st>>>(raw_k, h->n, key_s, h->Gp);
+        bsk::slice_bits_kernel<10, 80, false><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_k, h->n, key_s, h->Gp);
         if (int rc = check_launch("slice(key)")) return rc;
-        bsk::slice_bits_kernel<8, 64, false><<<sblocks, 256, 0, st>>>(raw_iv, h->n, iv_s, h->Gp);
+        bsk::slice_bits_kernel<8, 64, false><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_iv, h->n, iv_s, h->Gp);
         if (int rc = check_launch("slice(iv)")) return rc;
         const unsigned pblocks = unsigned((h->Gp + 127) / 128);
         bsk::grain_preclock_kernel<<<pblocks, 128, 0, st>>>(key_s, iv_s, h->state, h->Gp);
@@ -147,7 +147,7 @@ int run_init(bsrng_t* h, cudaStream_t st)
     case BSRNG_AES128_CTR: {
         // initial counter blocks sliced straight into the state rows (FIPS-197
         // bit order: bit 0 = MSB of byte 0); round keys from the one key.
-        bsk::slice_bits_kernel<16, 128, true><<<sblocks, 256, 0, st>>>(raw_iv, h->n, h->state, h->Gp);
+        bsk::slice_bits_kernel<16, 128, true><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_iv, h->n, h->state, h->Gp);
         if (int rc = check_launch("slice(ctr)")) return rc;
         bsk::aes::aes_key_expand_kernel<<<1, 32, 0, st>>>(raw_k, h->rk_dev);
         if (int rc = check_launch("aes_key_expand")) return rc;

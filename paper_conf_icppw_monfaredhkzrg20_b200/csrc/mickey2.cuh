@@ -158,12 +158,23 @@ __global__ void __launch_bounds__(128) m2_preclock_kernel(const uint32_t* __rest
     uint32_t r[100], s[100];
 #pragma unroll
     for (int i = 0; i < 100; ++i) r[i] = s[i] = 0u;
+    // 4 clocks per loop iteration (iv_bits is a multiple of 8): the S-register
+    // renaming then closes inside the body instead of costing ~100 moves/clock
 #pragma unroll 1
-    for (int i = 0; i < iv_bits; ++i) m2::clock_kg<true>(r, s, iv_s[uint64_t(i) * Gp + g]);
+    for (int i = 0; i < iv_bits; i += 4) {
+#pragma unroll
+        for (int u = 0; u < 4; ++u) m2::clock_kg<true>(r, s, iv_s[uint64_t(i + u) * Gp + g]);
+    }
 #pragma unroll 1
-    for (int i = 0; i < 80; ++i) m2::clock_kg<true>(r, s, key_s[uint64_t(i) * Gp + g]);
+    for (int i = 0; i < 80; i += 4) {
+#pragma unroll
+        for (int u = 0; u < 4; ++u) m2::clock_kg<true>(r, s, key_s[uint64_t(i + u) * Gp + g]);
+    }
 #pragma unroll 1
-    for (int i = 0; i < 100; ++i) m2::clock_kg<true>(r, s, 0u);
+    for (int i = 0; i < 100; i += 4) {
+#pragma unroll
+        for (int u = 0; u < 4; ++u) m2::clock_kg<true>(r, s, 0u);
+    }
 #pragma unroll
     for (int i = 0; i < 100; ++i) state[uint64_t(i) * Gp + g] = r[i];
 #pragma unroll
