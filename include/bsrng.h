@@ -158,7 +158,9 @@ int64_t bsrng_copy_state(const bsrng_t* h, uint32_t* host_out, uint64_t words);
  *                  1 = persistent, time-segmented work queue (default)
  *   "seg_clocks" : clocks per work item when sched = 1 (multiple of 32)
  *   "ctas_per_sm": resident CTAs per SM for the persistent grid
- *   "unroll"     : clocks per loop iteration of the clock loop (1, 2, 4, 8)
+ *   "unroll"     : clocks per loop iteration (MICKEY 2, 4, 8; Grain 8, 16, 32)
+ *   "rm_ws"      : ROW_MAJOR kernel: -1 auto, 1 warp-specialised (AES: block-
+ *                  lane), 0 plain
  * Returns BSRNG_OK or BSRNG_EINVAL for an unknown key/value.
  */
 int bsrng_set_option(bsrng_t* h, const char* key, int64_t value);

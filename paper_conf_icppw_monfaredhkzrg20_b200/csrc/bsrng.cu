@@ -90,7 +90,10 @@ struct bsrng {
     // Resident CTAs per SM; 0 = auto (launch_keystream / launch_aes).
     int opt_ctas_per_sm = 0;
     int opt_unroll = KS_U_DEFAULT;
-    int opt_rm_ws = 1;  // ROW_MAJOR through the warp-specialised compute/writer kernel
+    // ROW_MAJOR kernel choice: -1 = auto (MICKEY: warp-specialised compute/
+    // writer kernel; Grain: in-register transpose in the clock kernel; AES:
+    // block-lane kernel for calls of >= 32 blocks), 1 = specialised, 0 = plain
+    int opt_rm_ws = -1;
 };
 
 namespace {
@@ -198,7 +201,8 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
 
     // ROW_MAJOR default: warp-specialised compute/writer kernel (rowmajor_ws.cuh),
     // 8 warps per CTA of which 4 run the clock loop; always persistent.
-    const bool ws = LAYOUT == bsk::L_ROW_MAJOR && h->opt_rm_ws && h->opt_sched != 0;
+    const bool ws_pref = h->opt_rm_ws < 0 ? (C::U_DEFAULT != 32) : (h->opt_rm_ws != 0);
+    const bool ws = LAYOUT == bsk::L_ROW_MAJOR && ws_pref && h->opt_sched != 0;
     int block = KS_BLOCK, compute_warps = KS_BLOCK / 32;
     size_t smem = LAYOUT == bsk::L_ROW_MAJOR ? size_t(KS_BLOCK / 32) * bsk::RM_WARP_WORDS * 4 : 0;
     if (ws) {
@@ -639,7 +643,7 @@ int bsrng_set_option(bsrng_t* h, const char* key, int64_t value)
         if (!ok) return fail(BSRNG_EINVAL, "unroll must be %s", grain ? "8, 16 or 32" : "2, 4 or 8");
         h->opt_unroll = int(value);
     } else if (!strcmp(key, "rm_ws")) {
-        if (value != 0 && value != 1) return fail(BSRNG_EINVAL, "rm_ws must be 0 or 1");
+        if (value < -1 || value > 1) return fail(BSRNG_EINVAL, "rm_ws must be -1 (auto), 0 or 1");
         h->opt_rm_ws = int(value);
     } else if (!strcmp(key, "block")) {
         if (value != KS_BLOCK) return fail(BSRNG_EINVAL, "block=%lld not built (built: %d)", (long long)value, KS_BLOCK);

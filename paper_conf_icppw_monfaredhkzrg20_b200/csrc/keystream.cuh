@@ -132,7 +132,24 @@ __device__ __forceinline__ void rowmajor_store(const uint32_t* os, uint8_t* row0
 {
     uint8_t* p = row0 + col;
     const uint64_t align = reinterpret_cast<uintptr_t>(p) | row_bytes;
-    if (k_lo == 0 && k_hi == 7 && (align & 15) == 0) {
+    if (k_lo == 0 && k_hi == 7 && (align & 15) == 0 && nvalid == 32) {
+        // all shared-memory loads of 8 rows first, then their 16 stores, so a
+        // lone warp does not wait out each load -> store latency per row
+#pragma unroll 1
+        for (uint32_t q0 = 0; q0 < 32; q0 += 8) {
+            uint32_t v[8][8];
+#pragma unroll
+            for (int r = 0; r < 8; ++r)
+#pragma unroll
+                for (int k = 0; k < 8; ++k) v[r][k] = os[((q0 + r) * 8 + k) * 32];
+#pragma unroll
+            for (int r = 0; r < 8; ++r) {
+                uint4* d = reinterpret_cast<uint4*>(p + (q0 + r) * row_bytes);
+                __stcs(d, make_uint4(v[r][0], v[r][1], v[r][2], v[r][3]));
+                __stcs(d + 1, make_uint4(v[r][4], v[r][5], v[r][6], v[r][7]));
+            }
+        }
+    } else if (k_lo == 0 && k_hi == 7 && (align & 15) == 0) {
 #pragma unroll 4
         for (uint32_t q = 0; q < nvalid; ++q) {
             const uint32_t* src = os + q * 8 * 32;
