@@ -1,0 +1,126 @@
+"""GPU tests of the C ABI surface beyond single-cipher parity: edge sizes,
+tuning options (every variant must stay bit-exact), concurrent handles on
+separate streams, chunked host generation, and the 2^40 limit boundary."""
+import numpy as np
+import pytest
+
+import oracle
+from helpers import checksum, to_sliced
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+from paper_conf_icppw_monfaredhkzrg20_b200 import bsrng, inputs  # noqa: E402
+
+
+def _want(cipher, keys, ivs, bits, first_block=0):
+    if cipher == "mickey2":
+        return oracle.mickey2_keystream_batch(keys, ivs, 80, bits)
+    if cipher == "grain":
+        return oracle.grain_keystream_batch(keys, ivs, bits)
+    return oracle.aes128_ctr_keystream_batch(bytes(inputs.aes_key()), ivs, bits, first_block=first_block)
+
+
+def _gen(cipher, keys, ivs, **kw):
+    if cipher == "aes128ctr":
+        return bsrng.Generator(cipher, inputs.aes_key(), ivs, **kw)
+    return bsrng.Generator(cipher, keys, ivs, **kw)
+
+
+@pytest.mark.parametrize("cipher", ["mickey2", "grain", "aes128ctr"])
+def test_single_instance(cipher):
+    keys, ivs = inputs.make_inputs(cipher, 1)
+    want = _want(cipher, keys, ivs, 512)
+    g = _gen(cipher, keys, ivs)
+    assert np.array_equal(g.generate_host(512, "row_major"), want)
+    sl = _gen(cipher, keys, ivs).generate_host(512, "sliced")
+    assert np.array_equal(sl, to_sliced(want, msb_first=cipher != "grain"))
+    assert np.all((sl >> np.uint32(1)) == 0)
+
+
+@pytest.mark.parametrize("cipher", ["mickey2", "grain", "aes128ctr"])
+def test_zero_bits_is_noop(cipher):
+    keys, ivs = inputs.make_inputs(cipher, 40)
+    g = _gen(cipher, keys, ivs)
+    buf = torch.zeros(64, dtype=torch.uint8, device="cuda")
+    g.generate(buf, 0, "row_major")
+    assert g.bits_done == 0
+    assert np.array_equal(g.generate_host(256, "row_major"), _want(cipher, keys, ivs, 256))
+
+
+@pytest.mark.parametrize("cipher,opts", [
+    ("mickey2", {"unroll": 2}), ("mickey2", {"unroll": 8}), ("mickey2", {"sched": 0}),
+    ("mickey2", {"ctas_per_sm": 2}), ("mickey2", {"rm_ws": 0}), ("mickey2", {"rm_ws": 1, "seg_clocks": 512}),
+    ("grain", {"unroll": 8}), ("grain", {"unroll": 16}), ("grain", {"rm_ws": 1}), ("grain", {"sched": 0}),
+    ("grain", {"ctas_per_sm": 1, "seg_clocks": 256}),
+    ("aes128ctr", {"ctas_per_sm": 1}), ("aes128ctr", {"rm_ws": 0}), ("aes128ctr", {"seg_clocks": 4096}),
+])
+def test_options_stay_bit_exact(cipher, opts):
+    n, bits = 32 * 40 + 9, 8192
+    keys, ivs = inputs.make_inputs(cipher, n)
+    want = _want(cipher, keys, ivs, bits)
+    for layout in ("row_major", "sliced", "checksum"):
+        g = _gen(cipher, keys, ivs)
+        for k, v in opts.items():
+            g.set_option(k, v)
+        got = g.generate_host(bits, layout)
+        sl = to_sliced(want, msb_first=cipher != "grain")
+        if layout == "row_major":
+            assert np.array_equal(got, want), layout
+        elif layout == "sliced":
+            assert np.array_equal(got, sl), layout
+        else:
+            assert int(got[0]) == checksum(sl), layout
+
+
+def test_option_validation():
+    keys, ivs = inputs.make_inputs("grain", 32)
+    g = bsrng.Generator("grain", keys, ivs)
+    for k, v in (("unroll", 4), ("sched", 2), ("seg_clocks", 33), ("ctas_per_sm", 99), ("rm_ws", 5)):
+        with pytest.raises(bsrng.BsrngError) as e:
+            g.set_option(k, v)
+        assert e.value.code == bsrng.EINVAL
+
+
+def test_concurrent_handles_on_streams():
+    n, bits = 32 * 64, 2048
+    handles, outs, wants = [], [], []
+    streams = [torch.cuda.Stream() for _ in range(3)]
+    for i, cipher in enumerate(("mickey2", "grain", "aes128ctr")):
+        keys, ivs = inputs.make_inputs(cipher, n, seed=100 + i)
+        if cipher == "aes128ctr":
+            g = bsrng.Generator(cipher, inputs.aes_key(100 + i), ivs)
+            want = oracle.aes128_ctr_keystream_batch(bytes(inputs.aes_key(100 + i)), ivs, bits)
+        else:
+            g = bsrng.Generator(cipher, keys, ivs)
+            want = _want(cipher, keys, ivs, bits)
+        out = torch.empty(g.out_bytes(bits, "row_major"), dtype=torch.uint8, device="cuda")
+        handles.append(g)
+        outs.append(out)
+        wants.append(want)
+    for g, out, st in zip(handles, outs, streams):
+        g.generate(out, bits, "row_major", stream=st)
+    torch.cuda.synchronize()
+    for out, want in zip(outs, wants):
+        assert np.array_equal(out.cpu().numpy().reshape(n, bits // 8), want)
+
+
+def test_generate_host_chunks_rows():
+    """ROW_MAJOR host output larger than the 1 GiB device bounce buffer is
+    produced in column chunks (cudaMemcpy2D into the host rows)."""
+    n, bits = 1 << 20, 1 << 14  # 2 GiB of keystream
+    keys, ivs = inputs.make_inputs("grain", n)
+    g = bsrng.Generator("grain", keys, ivs)
+    rows = g.generate_host(bits, "row_major")
+    idx = np.array([0, 1, 12345, n - 1])
+    assert np.array_equal(rows[idx], oracle.grain_keystream_batch(keys[idx], ivs[idx], bits))
+
+
+def test_mickey_2_40_limit_boundary():
+    keys, ivs = inputs.make_inputs("mickey2", 32)
+    g = bsrng.Generator("mickey2", keys, ivs)
+    buf = torch.empty(8, dtype=torch.int64, device="cuda")
+    with pytest.raises(bsrng.BsrngError) as e:
+        g.generate(buf, (1 << 40) + 32, "checksum")
+    assert e.value.code == bsrng.ERANGE
+    assert g.bits_done == 0
