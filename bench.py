@@ -44,8 +44,11 @@ def lop3_per_bit(cipher, mode):
         return 327.0
     if cipher == "grain":
         return 38.0 if mode == "consume" else 37.0
+    if cipher == "lfsr128":
+        return 3.0 if mode == "consume" else 2.0
     return (17280.0 + (64.0 if mode == "consume" else 0.0)) / 128.0
-CIPHER_NAME = {"mickey2": "MICKEY 2.0", "grain": "Grain v1", "aes128ctr": "AES-128-CTR"}
+CIPHER_NAME = {"mickey2": "MICKEY 2.0", "grain": "Grain v1", "aes128ctr": "AES-128-CTR",
+               "lfsr128": "bitsliced LFSR-128 (Eq. 2)"}
 ALU_LANES_PER_SM_CLK = 64      # 4 SMSP x 16 lanes (alu pipe rt = 2 cycles/warp-instr)
 METRIC = "MICKEY 2.0 keystream Tb/s (1 and 8 B200); fraction of LOP3/HBM roofline"
 
@@ -66,7 +69,7 @@ def parse():
                         "c3 = configs[2]: 2^25 instances x 2^18 bits = 1 TiB total, split across GPUs (strong); "
                         "c4 = configs[3]: the paper's launch shape, 2^19 instances x 4416 clocks per GPU; "
                         "rekey = SURVEY NEXT-3: 2^22 short streams x 2^10 bits, key/IV setup dominates")
-    p.add_argument("--cipher", default="mickey2", choices=["mickey2", "grain", "aes128ctr"])
+    p.add_argument("--cipher", default="mickey2", choices=["mickey2", "grain", "aes128ctr", "lfsr128"])
     p.add_argument("--n", type=int, default=None, help="instances per GPU (c2) / in total (c3)")
     p.add_argument("--bits", type=int, default=None, help="keystream bits per instance per step")
     p.add_argument("--no-context", action="store_true", help="skip the ALU-peak / cuRAND microbenchmarks")
@@ -177,6 +180,8 @@ def oracle_sample(n_inst, bits, first=0, threads=None, cipher="mickey2"):
     t = time.perf_counter()
     if cipher == "grain":
         oracle.grain_keystream_batch(keys, ivs, bits, threads=threads)
+    elif cipher == "lfsr128":
+        oracle.lfsr128_keystream_batch(keys, bits, threads=threads)
     elif cipher == "aes128ctr":
         oracle.aes128_ctr_keystream_batch(bytes(inputs.aes_key()), ivs, bits // 128 * 128, threads=threads)
     else:

@@ -38,7 +38,9 @@ extern "C" {
 typedef enum {
     BSRNG_MICKEY2 = 1,     /* MICKEY 2.0, sec. 2.3.1, sec. 4.4   */
     BSRNG_GRAIN_V1 = 2,    /* Grain v1,   PAPER.md:339-357 sec. 2.3.3 (NEXT-1)   */
-    BSRNG_AES128_CTR = 3   /* AES-128-CTR, sec. 2.3.2 (NEXT-2)  */
+    BSRNG_AES128_CTR = 3,  /* AES-128-CTR, sec. 2.3.2 (NEXT-2)  */
+    BSRNG_LFSR128 = 4      /* bitsliced LFSR of PAPER.md:545-596 sec. 4.3 (NEXT-4):
+                              x^128+x^29+x^27+x^2+1, state = 16-byte key, no IV */
 } bsrng_cipher;
 
 /* Output layouts of bsrng_generate (sec. 4.5 leaves the
@@ -80,9 +82,11 @@ typedef struct bsrng bsrng_t;
  * bsrng_create -- allocate device state for n instances, slice their keys/IVs
  * and run the initialisation clocks (MICKEY: iv_bits + 80 + 100 CLOCK_KG with
  * mixing, spec [5]); synchronous on the legacy stream.
- *   keys: HOST, row-major uint8[n][key_bytes]   (MICKEY/Grain 10 B, AES 16 B)
+ *   keys: HOST, row-major uint8[n][key_bytes]   (MICKEY/Grain 10 B, LFSR 16 B;
+ *         AES-128-CTR: ONE 16-byte key shared by all instances)
  *   ivs : HOST, row-major uint8[n][iv_bytes]    (MICKEY 10 B = 80-bit IV, the
- *         paper's benchmark IV; Grain 8 B; AES 16 B counter)
+ *         paper's benchmark IV; Grain 8 B; AES 16 B initial
+ *         128-bit big-endian counter block; LFSR none: ivs may be NULL)
  *   n   : number of instances, >= 1 (padded internally to 32*ceil(n/32))
  * Ownership: inputs are copied; the caller keeps its buffers.
  */
@@ -91,7 +95,7 @@ bsrng_t* bsrng_create(bsrng_cipher cipher, const uint8_t* keys, const uint8_t* i
 /*
  * bsrng_create_ex -- as bsrng_create, plus:
  *   iv_bits          : MICKEY IV length in bits, 0..80, multiple of 8 (IV row
- *                      stride is still 10 B); Grain must be 64; AES 128.
+ *                      stride is still 10 B); Grain must be 64; AES 128; LFSR 0.
  *   first_instance_id: global id of instance 0 (must be a multiple of 32); used
  *                      only to make CHECKSUM shard-invariant.
  *   flags            : BSRNG_INPUT_HOST or BSRNG_INPUT_DEVICE.

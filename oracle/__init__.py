@@ -8,7 +8,8 @@ shares no code with it.
 The arithmetic lives in plain C -- ``mickey2_ref.c`` (bit-serial MICKEY 2.0,
 spec [5]), ``grain_ref.c`` (bit-serial Grain v1, spec [15],
 PAPER.md:898-899), ``aes_ref.c`` (byte-oriented AES-128 + CTR, FIPS-197 [35],
-PAPER.md:957-959) -- compiled here into ``liboracle.so`` with gcc and called
+PAPER.md:957-959), ``lfsr_ref.c`` (the paper's bitsliced-LFSR example, Eq. 2,
+PAPER.md:545-596) -- compiled here into ``liboracle.so`` with gcc and called
 through ctypes.  This module only marshals arguments.
 """
 from __future__ import annotations
@@ -21,7 +22,7 @@ from concurrent.futures import ThreadPoolExecutor
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-_SOURCES = ["mickey2_ref.c", "grain_ref.c", "aes_ref.c"]
+_SOURCES = ["mickey2_ref.c", "grain_ref.c", "aes_ref.c", "lfsr_ref.c"]
 _LIB_PATH = os.path.join(_HERE, "liboracle.so")
 _lib = None
 
@@ -67,6 +68,10 @@ def lib() -> ctypes.CDLL:
         L.ref_aes_sbox.restype = ctypes.c_uint8
         L.ref_aes128_ctr_keystream.argtypes = [u8p, u8p, ctypes.c_uint64, ctypes.c_uint64, u8p]
         L.ref_aes128_ctr_keystream.restype = None
+        L.ref_lfsr128_keystream.argtypes = [u8p, ctypes.c_uint64, u8p]
+        L.ref_lfsr128_keystream.restype = None
+        L.ref_lfsr128_clock.argtypes = [u8p]
+        L.ref_lfsr128_clock.restype = ctypes.c_int
         _lib = L
     return _lib
 
@@ -249,3 +254,36 @@ def aes128_ctr_keystream_batch(key: bytes, ctrs: np.ndarray, nbits: int, first_b
         with ThreadPoolExecutor(max_workers=threads) as ex:
             list(ex.map(one, range(n)))
     return out[:, : nbits // 8]
+
+
+# ------------------------------------------------------------- 128-bit LFSR
+def lfsr128_keystream(key: bytes, nbits: int) -> bytes:
+    k = _buf(key, 16)
+    out = np.zeros(max((nbits + 7) // 8, 1), dtype=np.uint8)
+    lib().ref_lfsr128_keystream(_p(k), nbits, _p(out))
+    return out[: (nbits + 7) // 8].tobytes()
+
+
+def lfsr128_clock(s: np.ndarray):
+    s = np.ascontiguousarray(s, dtype=np.uint8).copy()
+    z = lib().ref_lfsr128_clock(_p(s))
+    return s, z
+
+
+def lfsr128_keystream_batch(keys: np.ndarray, nbits: int, threads: int | None = None) -> np.ndarray:
+    keys = np.ascontiguousarray(keys, dtype=np.uint8)
+    n = keys.shape[0]
+    out = np.zeros((n, max((nbits + 7) // 8, 1)), dtype=np.uint8)
+    L = lib()
+
+    def one(i):
+        L.ref_lfsr128_keystream(_p(keys[i]), nbits, _p(out[i]))
+
+    threads = threads or os.cpu_count() or 1
+    if threads == 1 or n == 1:
+        for i in range(n):
+            one(i)
+    else:
+        with ThreadPoolExecutor(max_workers=threads) as ex:
+            list(ex.map(one, range(n)))
+    return out[:, : (nbits + 7) // 8]

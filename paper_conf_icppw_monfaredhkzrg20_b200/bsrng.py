@@ -16,15 +16,15 @@ from . import inputs as _inputs
 _PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_PKG, "libbsrng.so")
 
-MICKEY2, GRAIN_V1, AES128_CTR = 1, 2, 3
+MICKEY2, GRAIN_V1, AES128_CTR, LFSR128 = 1, 2, 3, 4
 ROW_MAJOR, SLICED, CHECKSUM = 0, 1, 2
 INPUT_HOST, INPUT_DEVICE = 0, 1
 OK, EINVAL, ENOMEM, ECUDA, ERANGE, EUNSUPPORTED = 0, -1, -2, -3, -4, -5
 
-CIPHERS = {"mickey2": MICKEY2, "grain": GRAIN_V1, "aes128ctr": AES128_CTR}
+CIPHERS = {"mickey2": MICKEY2, "grain": GRAIN_V1, "aes128ctr": AES128_CTR, "lfsr128": LFSR128}
 LAYOUTS = {"row_major": ROW_MAJOR, "sliced": SLICED, "checksum": CHECKSUM}
-NSTATE = {MICKEY2: 200, GRAIN_V1: 160, AES128_CTR: 128}
-DEFAULT_IV_BITS = {MICKEY2: 80, GRAIN_V1: 64, AES128_CTR: 128}
+NSTATE = {MICKEY2: 200, GRAIN_V1: 160, AES128_CTR: 128, LFSR128: 128}
+DEFAULT_IV_BITS = {MICKEY2: 80, GRAIN_V1: 64, AES128_CTR: 128, LFSR128: 0}
 
 SYMBOLS = [
     "bsrng_create", "bsrng_create_ex", "bsrng_rekey", "bsrng_generate", "bsrng_generate_host",
@@ -137,6 +137,8 @@ class Generator:
         self.cipher = CIPHERS[cipher] if isinstance(cipher, str) else int(cipher)
         self.iv_bits = DEFAULT_IV_BITS.get(self.cipher, 0) if iv_bits is None else int(iv_bits)
         kp, kdev = _ptr(keys)
+        if ivs is not None and getattr(ivs, "size", 1) == 0:
+            ivs = None  # no IV (LFSR)
         vp, vdev = _ptr(ivs)
         # AES-128-CTR: ONE key for all instances, n = number of counter blocks
         rows = ivs if self.cipher == AES128_CTR else keys
@@ -179,6 +181,8 @@ class Generator:
     # -- operations -------------------------------------------------------
     def rekey(self, keys, ivs, stream=None):
         kp, kdev = _ptr(keys)
+        if ivs is not None and getattr(ivs, "size", 1) == 0:
+            ivs = None
         vp, _ = _ptr(ivs)
         self._keep = (keys, ivs)
         _check(lib().bsrng_rekey(self._h, kp, vp, INPUT_DEVICE if kdev else INPUT_HOST,

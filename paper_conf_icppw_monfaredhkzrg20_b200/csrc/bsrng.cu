@@ -20,6 +20,7 @@
 #include "keystream.cuh"
 #include "aes.cuh"
 #include "grain.cuh"
+#include "lfsr.cuh"
 #include "mickey2.cuh"
 #include "rowmajor_ws.cuh"
 
@@ -104,6 +105,7 @@ int nstate_of(bsrng_cipher c)
     case BSRNG_MICKEY2: return bsk::Mickey2::NSTATE;
     case BSRNG_GRAIN_V1: return bsk::Grain::NSTATE;
     case BSRNG_AES128_CTR: return bsk::aes::NSTATE;
+    case BSRNG_LFSR128: return bsk::Lfsr128::NSTATE;
     default: return 0;
     }
 }
@@ -159,6 +161,16 @@ int run_init(bsrng_t* h, cudaStream_t st)
         cudaError_t e = cudaMemcpyAsync(&h->rk, h->rk_dev, sizeof(h->rk), cudaMemcpyDeviceToHost, st);
         if (e == cudaSuccess) e = cudaStreamSynchronize(st);
         if (e != cudaSuccess) return fail(BSRNG_ECUDA, "round keys: %s", cudaGetErrorString(e));
+        (void)key_s;
+        (void)iv_s;
+        return BSRNG_OK;
+    }
+    case BSRNG_LFSR128: {
+        // the state IS the key: 128 bits, MSB-first, sliced straight into rows 0..127
+        bsk::slice_bits_kernel<16, 128, true><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_k, h->n, h->state, h->Gp);
+        if (int rc = check_launch("slice(key)")) return rc;
+        cudaError_t e = cudaMemsetAsync(h->state + uint64_t(bsk::Lfsr128::NSTATE) * h->Gp, 0, h->Gp * 4, st);
+        if (e != cudaSuccess) return fail(BSRNG_ECUDA, "memset: %s", cudaGetErrorString(e));
         (void)key_s;
         (void)iv_s;
         return BSRNG_OK;
@@ -441,6 +453,10 @@ bsrng_t* bsrng_create_ex(bsrng_cipher cipher, const uint8_t* keys, const uint8_t
     if (n == 0) { fail(BSRNG_EINVAL, "n_instances == 0"); return nullptr; }
     if (first_instance_id % 32) { fail(BSRNG_EINVAL, "first_instance_id must be a multiple of 32"); return nullptr; }
     if (flags & ~uint32_t(BSRNG_INPUT_DEVICE)) { fail(BSRNG_EINVAL, "unknown flags 0x%x", flags); return nullptr; }
+    if (cipher == BSRNG_LFSR128 && iv_bits != 0) {
+        fail(BSRNG_EINVAL, "LFSR iv_bits=%u must be 0 (the state is the key)", iv_bits);
+        return nullptr;
+    }
     if (cipher == BSRNG_GRAIN_V1 && iv_bits != 64) {
         fail(BSRNG_EINVAL, "Grain v1 iv_bits=%u must be 64", iv_bits);
         return nullptr;
@@ -467,12 +483,12 @@ bsrng_t* bsrng_create_ex(bsrng_cipher cipher, const uint8_t* keys, const uint8_t
     h->Gp = h->units * 32;
     h->first_instance = first_instance_id;
     h->iv_bits = iv_bits;
-    const bool aes = cipher == BSRNG_AES128_CTR;
-    h->key_bytes = aes ? 16 : 10;
-    h->iv_bytes = cipher == BSRNG_GRAIN_V1 ? 8 : aes ? 16 : 10;
+    const bool aes = cipher == BSRNG_AES128_CTR, lfsr = cipher == BSRNG_LFSR128;
+    h->key_bytes = (aes || lfsr) ? 16 : 10;
+    h->iv_bytes = cipher == BSRNG_GRAIN_V1 ? 8 : aes ? 16 : lfsr ? 0 : 10;
     h->key_rows = aes ? 1 : h->n;
     const int ns = nstate_of(cipher);
-    const uint64_t sl_words = aes ? 1 : uint64_t(h->key_bytes + h->iv_bytes) * 8 * h->Gp;
+    const uint64_t sl_words = (aes || lfsr) ? 1 : uint64_t(h->key_bytes + h->iv_bytes) * 8 * h->Gp;
     if (cudaMalloc(&h->state, uint64_t(ns + 1) * h->Gp * 4) != cudaSuccess ||
         cudaMalloc(&h->sliced, sl_words * 4) != cudaSuccess ||
         cudaMalloc(&h->raw, h->key_rows * h->key_bytes + h->n * h->iv_bytes) != cudaSuccess ||
@@ -501,7 +517,7 @@ bsrng_t* bsrng_create_ex(bsrng_cipher cipher, const uint8_t* keys, const uint8_t
 
 bsrng_t* bsrng_create(bsrng_cipher cipher, const uint8_t* keys, const uint8_t* ivs, uint64_t n)
 {
-    const uint32_t ivb = cipher == BSRNG_GRAIN_V1 ? 64 : cipher == BSRNG_AES128_CTR ? 128 : 80;
+    const uint32_t ivb = cipher == BSRNG_GRAIN_V1 ? 64 : cipher == BSRNG_AES128_CTR ? 128 : cipher == BSRNG_LFSR128 ? 0 : 80;
     return bsrng_create_ex(cipher, keys, ivs, ivb, n, 0, BSRNG_INPUT_HOST, nullptr);
 }
 
@@ -538,6 +554,7 @@ int bsrng_generate(bsrng_t* h, void* out, uint64_t bits, bsrng_layout layout, vo
     switch (h->cipher) {
     case BSRNG_MICKEY2: rc = dispatch_layout<bsk::Mickey2>(h, out, bits, layout, st); break;
     case BSRNG_GRAIN_V1: rc = dispatch_layout<bsk::Grain>(h, out, bits, layout, st); break;
+    case BSRNG_LFSR128: rc = dispatch_layout<bsk::Lfsr128>(h, out, bits, layout, st); break;
     case BSRNG_AES128_CTR:
         rc = layout == BSRNG_ROW_MAJOR ? (bits >= 4096 && h->opt_rm_ws ? launch_aes_rowmajor_lanes(h, out, bits, st)
                                                                        : launch_aes<bsk::L_ROW_MAJOR>(h, out, bits, st))
@@ -637,7 +654,7 @@ int bsrng_set_option(bsrng_t* h, const char* key, int64_t value)
         if (value < 0 || value > 32) return fail(BSRNG_EINVAL, "ctas_per_sm out of range");
         h->opt_ctas_per_sm = int(value);
     } else if (!strcmp(key, "unroll")) {
-        const bool grain = h->cipher == BSRNG_GRAIN_V1;
+        const bool grain = h->cipher == BSRNG_GRAIN_V1 || h->cipher == BSRNG_LFSR128;
         const bool ok = value == 0 || (grain ? (value == 8 || value == 16 || value == 32)
                                              : (value == 2 || value == 4 || value == 8));
         if (!ok) return fail(BSRNG_EINVAL, "unroll must be %s", grain ? "8, 16 or 32" : "2, 4 or 8");

@@ -1,0 +1,49 @@
+// lfsr.cuh -- the paper's bitsliced LFSR, sm_100a.
+//
+// PAPER.md:578-596 (sec. 4.3, Fig. 8): "the bitsliced LFSR implementation with
+// column-major representation ... executed by a single thread ... the 32 x k
+// number of costly bit-wise XOR operations is reduced to k number of full-width
+// XOR operations ... the costly bit-level shift operations are replaced by ...
+// register swapping".  Polynomial (reading L1): p(x) = x^128 + x^29 + x^27 +
+// x^2 + 1, primitive; Fibonacci form s_{t+128} = s_{t+29} ^ s_{t+27} ^ s_{t+2}
+// ^ s_t, output z_t = s_t.  Per clock: 2 LOP3 for 32 keystream bits (k = 4
+// taps); the shift is renaming, closed by 128/U moves per clock (FMA pipe).
+// With so little logic the materialised keystream is bound by HBM writes --
+// this workload exercises the output path at the memory roofline.
+#pragma once
+#include <cstdint>
+
+#include "bitslice.cuh"
+
+namespace bsk {
+
+struct Lfsr128 {
+    static constexpr int NSTATE = 128;
+    static constexpr bool MSB_FIRST = true;
+    static constexpr int U_DEFAULT = 32, U_ALT0 = 8, U_ALT1 = 16;
+    uint32_t s[128];
+
+    __device__ __forceinline__ void load(const uint32_t* st, uint64_t Gp, uint64_t g)
+    {
+        const uint32_t* p = opaque(st + g);
+#pragma unroll
+        for (int i = 0; i < 128; ++i) s[i] = __ldcg(p + uint64_t(i) * Gp);
+    }
+    __device__ __forceinline__ void store(uint32_t* st, uint64_t Gp, uint64_t g) const
+    {
+        uint32_t* p = opaque(st + g);
+#pragma unroll
+        for (int i = 0; i < 128; ++i) __stcg(p + uint64_t(i) * Gp, s[i]);
+    }
+    __device__ __forceinline__ uint32_t z() const { return s[0]; }
+    __device__ __forceinline__ uint32_t z_acc(uint32_t acc) const { return acc ^ s[0]; }
+    __device__ __forceinline__ void clock()
+    {
+        const uint32_t fb = lop3<0x96u>(lop3<0x96u>(s[29], s[27], s[2]), s[0], 0u);
+#pragma unroll
+        for (int i = 0; i < 127; ++i) s[i] = s[i + 1];
+        s[127] = fb;
+    }
+};
+
+}  // namespace bsk

@@ -20,6 +20,7 @@ cipher         key                              IV / counter
 MICKEY 2.0     LE(x0) || LE(x1)[0:2]  (10 B)    LE(x2) || LE(x3)[0:2]  (10 B)
 Grain v1       LE(x0) || LE(x1)[0:2]  (10 B)    LE(x2)                 (8 B)
 AES-128-CTR    LE(x0) || LE(x1)       (16 B)    LE(x2) || LE(x3)       (16 B)
+LFSR-128       LE(x0) || LE(x1)       (16 B)    none
 =============  ==============================  ==============================
 
 AES-128-CTR runs every instance under ONE key ("different
@@ -36,8 +37,8 @@ M1 = np.uint64(0xBF58476D1CE4E5B9)
 M2 = np.uint64(0x94D049BB133111EB)
 DEFAULT_SEED = 0x5EED2020
 
-KEY_BYTES = {"mickey2": 10, "grain": 10, "aes128ctr": 16}
-IV_BYTES = {"mickey2": 10, "grain": 8, "aes128ctr": 16}
+KEY_BYTES = {"mickey2": 10, "grain": 10, "aes128ctr": 16, "lfsr128": 16}
+IV_BYTES = {"mickey2": 10, "grain": 8, "aes128ctr": 16, "lfsr128": 0}
 
 
 def fmix64(z: np.ndarray) -> np.ndarray:
