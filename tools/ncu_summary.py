@@ -38,8 +38,13 @@ UNIT_SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12
 
 
 def raw_metrics(rep):
-    txt = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    if rep.endswith(".csv"):
+        txt = open(rep).read()
+    else:
+        txt = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(txt)))
+    if len(rows) < 3:
+        return []
     hdr, units = rows[0], rows[1]
     out = []
     for row in rows[2:]:
@@ -91,9 +96,12 @@ def main():
 
     traffic = {}
     for rep in sorted(os.listdir(src)):
-        if not rep.endswith(".ncu-rep"):
+        if rep.endswith(".ncu-rep"):
+            name = rep[:-8]
+        elif rep.endswith("_raw.csv"):
+            name = rep[:-8]
+        else:
             continue
-        name = rep[:-8]
         ms = raw_metrics(os.path.join(src, rep))
         if not ms:
             continue
@@ -104,8 +112,9 @@ def main():
             for k in KEYS:
                 if k in m:
                     w.writerow([k, m[k][0], m[k][1]])
-        log = open(os.path.join(src, f"ncu_{name.replace('ks_', '')}.log")).read() \
-            if os.path.exists(os.path.join(src, f"ncu_{name.replace('ks_', '')}.log")) else ""
+        logf = [os.path.join(src, f"ncu_{name}.log"), os.path.join(src, f"ncu_{name.replace('ks_', '')}.log")]
+        logf = [f for f in logf if os.path.exists(f)]
+        log = open(logf[0]).read() if logf else ""
         lines.append(f"\n## `{name}` — {m.get('Kernel Name', ('?', ''))[0][:100]}\n")
         argline = [ln for ln in log.splitlines() if ln.startswith("done Namespace")]
         if argline:
@@ -121,11 +130,12 @@ def main():
         f.write("\n".join(lines) + "\n")
     if "ks_consume" in traffic:
         t = traffic["ks_consume"]
+        t = dict(t)
         json.dump({"mode": "consume", "n": 1 << 22,
                    "dram_bytes_per_launch": t["dram_read"] + t["dram_write"],
                    "note": ("ncu --set full capture of keystream_kernel<CHECKSUM> at n=2^22, 2^16 bits "
-                            f"({tag}); the persistent launch has the same 5 segments (state carry "
-                            "5 x 200 MiB R+W) at the bench's 2^20 bits, so bytes per launch match"),
+                            f"({tag}); at the bench's 2^20 bits the launch has the same work items (one per "
+                            "warp-unit, state carry 100 MiB in + 100 MiB out), so bytes per launch match"),
                    "captures": traffic}, open(os.path.join(prof, "keystream_traffic.json"), "w"), indent=1)
     print("\n".join(lines))
 
