@@ -82,6 +82,8 @@ def parse():
     p.add_argument("--sched", type=int, default=None)
     p.add_argument("--seg-clocks", type=int, default=None)
     p.add_argument("--ctas-per-sm", type=int, default=None)
+    p.add_argument("--opt", action="append", default=[], metavar="KEY=VALUE",
+                   help="extra bsrng_set_option knob (A/B runs; defaults are the tuned ones)")
     return p.parse_args()
 
 
@@ -306,6 +308,9 @@ def run_ours(args, rank, world, local_rank):
     for k, v in (("sched", args.sched), ("seg_clocks", args.seg_clocks), ("ctas_per_sm", args.ctas_per_sm)):
         if v is not None:
             g.set_option(k, v)
+    for kv in args.opt:
+        k, v = kv.split("=")
+        g.set_option(k, int(v))
     cs_out = torch.zeros(1, dtype=torch.int64, device=dev)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
 

@@ -165,6 +165,18 @@ int64_t bsrng_copy_state(const bsrng_t* h, uint32_t* host_out, uint64_t words);
  *   "unroll"     : clocks per loop iteration (MICKEY 2, 4, 8; Grain 8, 16, 32)
  *   "rm_ws"      : ROW_MAJOR kernel: -1 auto, 1 warp-specialised (AES: block-
  *                  lane), 0 plain
+ *   "rm_slots"   : ROW_MAJOR plain kernel: 32-clock blocks staged per row
+ *                  before a flush, 8 (one 32 B sector per row) or 4 (16 B,
+ *                  half the shared memory); 0 = auto
+ *   "rm_zreg"    : ROW_MAJOR plain kernel with 32 clocks per iteration: keep
+ *                  the z block in registers (1, default) or stage it in
+ *                  shared memory (0)
+ *   "rm_tmem"    : ROW_MAJOR plain kernel: stage the row segments in tensor
+ *                  memory (TMEM, 256 columns per CTA) instead of shared
+ *                  memory (1); default 0 (measured slower)
+ *   "init_fused" : MICKEY / Grain create/rekey: slicing fused into the
+ *                  initialisation kernel (1, default) or the separate
+ *                  slice_bits + preclock kernels (0)
  * Returns BSRNG_OK or BSRNG_EINVAL for an unknown key/value.
  */
 int bsrng_set_option(bsrng_t* h, const char* key, int64_t value);

@@ -31,36 +31,41 @@ __device__ __forceinline__ uint32_t lop3(uint32_t a, uint32_t b, uint32_t c)
 //           (MICKEY, spec [5]), (byte[b/8] >> (b%8)) & 1 otherwise (Grain)
 // Instances >= n (padding) get all-zero bytes.
 // ---------------------------------------------------------------------------
-// Block = 32 warps = 32 consecutive groups; the ballot words are staged in
-// shared memory as [bit][group] and written out as one coalesced 128 B row
-// segment per bit (per-warp 4-byte stores strided by Gp were 20x slower).
-constexpr int SLICE_BLOCK = 1024;
+// Block = SLICE_GROUPS warps = that many consecutive groups; the ballot words
+// are staged in shared memory as [bit][group] and written out as one 32 B DRAM
+// sector per bit (per-warp 4-byte stores strided by Gp were 20x slower).  The
+// first version used 1024-thread blocks (32 groups, one 128 B segment per
+// bit): one resident block per SM left the loads' latency exposed (120 us per
+// 2^22 keys); 256-thread blocks keep 8 blocks in flight per SM.
+constexpr int SLICE_GROUPS = 8;
+constexpr int SLICE_BLOCK = 32 * SLICE_GROUPS;
 
 template <int NBYTES, int NBITS, bool MSB>
 __global__ void __launch_bounds__(SLICE_BLOCK) slice_bits_kernel(const uint8_t* __restrict__ raw,
                                                                  uint64_t n, uint32_t* __restrict__ out,
                                                                  uint64_t Gp)
 {
-    __shared__ uint32_t tile[NBITS][33];
+    __shared__ uint32_t tile[NBITS][SLICE_GROUPS];
     const uint32_t wib = threadIdx.x >> 5;
     const uint32_t lane = threadIdx.x & 31u;
-    const uint64_t g0 = uint64_t(blockIdx.x) * 32u;  // first group of this block
+    const uint64_t g0 = uint64_t(blockIdx.x) * SLICE_GROUPS;  // first group of this block
     const uint64_t warp = g0 + wib;
     if (warp < Gp) {  // warp-uniform
         const uint64_t inst = warp * 32u + lane;
-        uint8_t b[NBYTES];
+        const uint8_t* src = raw + (inst < n ? inst : 0) * NBYTES;
+        uint32_t b[NBYTES];
 #pragma unroll
-        for (int i = 0; i < NBYTES; ++i) b[i] = (inst < n) ? raw[inst * NBYTES + i] : uint8_t(0);
+        for (int i = 0; i < NBYTES; ++i) b[i] = (inst < n) ? uint32_t(__ldg(src + i)) : 0u;
 #pragma unroll
         for (int bit = 0; bit < NBITS; ++bit) {
             const uint32_t v = MSB ? (b[bit >> 3] >> (7 - (bit & 7))) & 1u : (b[bit >> 3] >> (bit & 7)) & 1u;
             const uint32_t w = __ballot_sync(0xffffffffu, v);
-            if (lane == uint32_t(bit & 31)) tile[bit][wib] = w;
+            if (lane == 0) tile[bit][wib] = w;
         }
     }
     __syncthreads();
-    for (uint32_t idx = threadIdx.x; idx < uint32_t(NBITS) * 32u; idx += SLICE_BLOCK) {
-        const uint32_t bit = idx >> 5, gw = idx & 31u;
+    for (uint32_t idx = threadIdx.x; idx < uint32_t(NBITS) * SLICE_GROUPS; idx += SLICE_BLOCK) {
+        const uint32_t bit = idx / SLICE_GROUPS, gw = idx % SLICE_GROUPS;
         if (g0 + gw < Gp) out[uint64_t(bit) * Gp + g0 + gw] = tile[bit][gw];
     }
 }
@@ -122,6 +127,68 @@ __device__ __forceinline__ void bt_transpose16(uint32_t (&x)[16])
 #pragma unroll
     for (int r = 0; r < 16; ++r)
         if ((r & 1) == 0) bt_stage<1, 0x55555555u>(x[r], x[r + 1]);
+}
+
+// ---------------------------------------------------------------------------
+// Per-thread key/IV slicing for fused init kernels (SURVEY step a-1 inside
+// a-2).  Thread = one group of 32 instances, as in the clock loop.  `p` =
+// the group's 32 byte strings (32*NBYTES bytes, 16 B aligned, zero-padded past
+// n).  For each 32-bit chunk c the thread builds A[j] = bytes 4c..4c+3 of
+// instance j (big-endian if MSB, so string bit 32c+t is A bit 31-t; else
+// little-endian, bit 32c+t = A bit t), transposes the 32x32 block in
+// registers (bt_transpose16: B[r] bit j = A[j] bit r) and hands every slice
+// word to put(bit, word): bit 32c+31-r (MSB) or 32c+r (LSB).  The group's
+// bytes are read with 16 B loads straight into registers (no smem staging).
+// ---------------------------------------------------------------------------
+template <int NBYTES, int NBITS, bool MSB, class Put>
+__device__ __forceinline__ void slice_group32(const uint8_t* __restrict__ p, Put&& put)
+{
+    static_assert((32 * NBYTES) % 16 == 0, "group block must be whole 16 B vectors");
+    constexpr int NW = 32 * NBYTES / 4;
+    uint32_t raw[NW + 1];
+    const uint4* src = reinterpret_cast<const uint4*>(p);
+#pragma unroll
+    for (int i = 0; i < NW / 4; ++i) {
+        const uint4 v = __ldcs(src + i);
+        raw[4 * i] = v.x;
+        raw[4 * i + 1] = v.y;
+        raw[4 * i + 2] = v.z;
+        raw[4 * i + 3] = v.w;
+    }
+    raw[NW] = 0u;  // straddle guard for the last instance's final chunk
+    constexpr int NCHUNK = (NBITS + 31) / 32;
+#pragma unroll
+    for (int c = 0; c < NCHUNK; ++c) {
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            // rows r = 16h + q; skip halves whose bits are all >= NBITS
+            const int lo_bit = MSB ? 32 * c + 31 - (16 * h + 15) : 32 * c + 16 * h;
+            if (lo_bit >= NBITS) continue;
+            uint32_t x[16];
+#pragma unroll
+            for (int q = 0; q < 16; ++q) {
+                uint32_t a2[2];
+#pragma unroll
+                for (int e = 0; e < 2; ++e) {
+                    const int j = q + 16 * e;
+                    const int bo = NBYTES * j + 4 * c;
+                    const int w0 = bo / 4, off = bo % 4;
+                    const uint32_t sel = MSB ? ((uint32_t(off) << 12) | (uint32_t(off + 1) << 8) |
+                                                (uint32_t(off + 2) << 4) | uint32_t(off + 3))
+                                             : ((uint32_t(off + 3) << 12) | (uint32_t(off + 2) << 8) |
+                                                (uint32_t(off + 1) << 4) | uint32_t(off));
+                    a2[e] = __byte_perm(raw[w0], off ? raw[w0 + 1] : 0u, sel);
+                }
+                x[q] = __byte_perm(a2[0], a2[1], h == 0 ? 0x5410 : 0x7632);
+            }
+            bt_transpose16(x);  // x[q] = B[16h + q]
+#pragma unroll
+            for (int q = 0; q < 16; ++q) {
+                const int bit = MSB ? 32 * c + 31 - (16 * h + q) : 32 * c + 16 * h + q;
+                if (bit < NBITS) put(bit, x[q]);
+            }
+        }
+    }
 }
 
 // Hide a pointer's provenance from the optimiser (no code emitted beyond a

@@ -79,7 +79,8 @@ struct bsrng {
     uint64_t bits_done = 0;
     uint32_t* state = nullptr;   // [NSTATE + 1][Gp]
     uint32_t* sliced = nullptr;  // key [KB][Gp] then iv [IVB][Gp]
-    uint8_t* raw = nullptr;      // keys [n][key_bytes] then ivs [n][iv_bytes]
+    uint8_t* raw = nullptr;      // keys [n][key_bytes] then ivs [n][iv_bytes] at raw + iv_off
+    uint64_t iv_off = 0;         // MICKEY: both regions padded to Gp*32*10 B (zeroed), 16 B aligned
     uint32_t* sched = nullptr;   // [1 + units]: ticket, flags; then [32] scratch
     uint8_t* bounce = nullptr;   // generate_host staging
     uint32_t* rk_dev = nullptr;  // AES: round-key masks written by the key-expansion kernel
@@ -95,6 +96,14 @@ struct bsrng {
     // writer kernel; Grain: in-register transpose in the clock kernel; AES:
     // block-lane kernel for calls of >= 32 blocks), 1 = specialised, 0 = plain
     int opt_rm_ws = -1;
+    // ROW_MAJOR sector-staging slots per row (4 or 8); 0 = auto.
+    int opt_rm_slots = 0;
+    // ROW_MAJOR, U = 32: z block in registers (1) or staged in smem (0).
+    int opt_rm_zreg = 1;
+    // ROW_MAJOR plain kernel: stage row segments in TMEM (1) or smem (0).
+    int opt_rm_tmem = 0;
+    // MICKEY / Grain init: fused slicing + preclock kernel (1) or slice kernels + preclock (0).
+    int opt_init_fused = 1;
 };
 
 namespace {
@@ -125,10 +134,24 @@ int run_init(bsrng_t* h, cudaStream_t st)
     uint32_t* key_s = h->sliced;
     uint32_t* iv_s = h->sliced + kbits * h->Gp;
     const uint8_t* raw_k = h->raw;
-    const uint8_t* raw_iv = h->raw + h->key_rows * h->key_bytes;
-    const unsigned sblocks = unsigned((h->Gp + 31) / 32);  // 32 groups per 1024-thread block
+    const uint8_t* raw_iv = h->raw + h->iv_off;
+    const unsigned sblocks = unsigned((h->Gp + bsk::SLICE_GROUPS - 1) / bsk::SLICE_GROUPS);
     switch (h->cipher) {
     case BSRNG_MICKEY2: {
+        if (h->opt_init_fused) {
+            // one kernel: slicing in shared memory + the 260 mixing clocks
+            const unsigned blocks = unsigned((h->Gp + bsk::M2I_BLOCK - 1) / bsk::M2I_BLOCK);
+            static bool attr = false;
+            if (!attr) {
+                cudaError_t e = cudaFuncSetAttribute(bsk::m2_init_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                     int(bsk::M2I_SMEM_BYTES));
+                if (e != cudaSuccess) return fail(BSRNG_ECUDA, "smem attribute: %s", cudaGetErrorString(e));
+                attr = true;
+            }
+            bsk::m2_init_kernel<<<blocks, bsk::M2I_BLOCK, bsk::M2I_SMEM_BYTES, st>>>(raw_k, raw_iv, int(h->iv_bits),
+                                                                                       h->state, h->Gp);
+            return check_launch("m2_init");
+        }
         bsk::slice_bits_kernel<10, 80, true><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_k, h->n, key_s, h->Gp);
         if (int rc = check_launch("slice(key)")) return rc;
         bsk::slice_bits_kernel<10, 80, true><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_iv, h->n, iv_s, h->Gp);
@@ -141,6 +164,11 @@ int run_init(bsrng_t* h, cudaStream_t st)
     }
     case BSRNG_GRAIN_V1: {
         // spec [15]: key and IV bits are taken LSB-first from their bytes
+        if (h->opt_init_fused) {
+            const unsigned blocks = unsigned((h->Gp + 127) / 128);
+            bsk::grain_init_kernel<<<blocks, 128, 0, st>>>(raw_k, raw_iv, h->state, h->Gp);
+            return check_launch("grain_init");
+        }
         bsk::slice_bits_kernel<10, 80, false><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_k, h->n, key_s, h->Gp);
         if (int rc = check_launch("slice(key)")) return rc;
         bsk::slice_bits_kernel<8, 64, false><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_iv, h->n, iv_s, h->Gp);
@@ -184,18 +212,47 @@ int copy_inputs(bsrng_t* h, const uint8_t* keys, const uint8_t* ivs, uint32_t fl
     const size_t kb = size_t(h->key_rows) * h->key_bytes, vb = size_t(h->n) * h->iv_bytes;
     const cudaMemcpyKind kind = (flags & BSRNG_INPUT_DEVICE) ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
     cudaError_t e = cudaMemcpyAsync(h->raw, keys, kb, kind, st);
-    if (e == cudaSuccess && vb) e = cudaMemcpyAsync(h->raw + kb, ivs, vb, kind, st);
+    if (e == cudaSuccess && vb) e = cudaMemcpyAsync(h->raw + h->iv_off, ivs, vb, kind, st);
     if (e != cudaSuccess) return fail(BSRNG_ECUDA, "key/iv copy failed: %s", cudaGetErrorString(e));
     return BSRNG_OK;
+}
+
+// Kernel instance for the handle's unroll option and ROW_MAJOR staging slots.
+template <class C, int LAYOUT, int SLOTS, bool ZREG = true, bool TMEM = false>
+auto pick_keystream_kernel(const bsrng_t* h, int* U)
+{
+    auto kern = &bsk::keystream_kernel<C, LAYOUT, C::U_DEFAULT, KS_BLOCK, SLOTS, ZREG, TMEM>;
+    *U = C::U_DEFAULT;
+    if (h->opt_unroll == C::U_ALT0)
+        kern = &bsk::keystream_kernel<C, LAYOUT, C::U_ALT0, KS_BLOCK, SLOTS, true, TMEM>, *U = C::U_ALT0;
+    if (h->opt_unroll == C::U_ALT1)
+        kern = &bsk::keystream_kernel<C, LAYOUT, C::U_ALT1, KS_BLOCK, SLOTS, true, TMEM>, *U = C::U_ALT1;
+    return kern;
 }
 
 template <class C, int LAYOUT>
 int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
 {
-    using K = decltype(&bsk::keystream_kernel<C, LAYOUT, C::U_DEFAULT, KS_BLOCK>);
-    K kern = &bsk::keystream_kernel<C, LAYOUT, C::U_DEFAULT, KS_BLOCK>;
-    if (h->opt_unroll == C::U_ALT0) kern = &bsk::keystream_kernel<C, LAYOUT, C::U_ALT0, KS_BLOCK>;
-    if (h->opt_unroll == C::U_ALT1) kern = &bsk::keystream_kernel<C, LAYOUT, C::U_ALT1, KS_BLOCK>;
+    // ROW_MAJOR row-segment staging: 8 slots (whole 32 B sectors, default) or
+    // 4 (16 B, half the shared memory; ncu: L2 then fetches and re-evicts the
+    // half-written sectors, ~3x the algorithmic DRAM traffic).
+    int slots = h->opt_rm_slots ? h->opt_rm_slots : 8;
+    if (LAYOUT != bsk::L_ROW_MAJOR) slots = 8;
+    // U = 32 loops keep the 32-clock z block in registers (zreg) or stage it
+    // in shared memory one word per clock (fewer live registers).
+    const bool zreg = LAYOUT != bsk::L_ROW_MAJOR || h->opt_rm_zreg != 0;
+    // TMEM: stage the row segments in tensor memory instead of shared memory
+    const bool tmem = LAYOUT == bsk::L_ROW_MAJOR && h->opt_rm_tmem > 0;
+    int U = 0;
+    auto kern = pick_keystream_kernel<C, LAYOUT, 8>(h, &U);
+    if (tmem) {
+        kern = zreg ? pick_keystream_kernel<C, LAYOUT, 8, true, true>(h, &U)
+                    : pick_keystream_kernel<C, LAYOUT, 8, false, true>(h, &U);
+    } else if (LAYOUT == bsk::L_ROW_MAJOR) {
+        if (slots == 4 && zreg) kern = pick_keystream_kernel<C, LAYOUT, 4>(h, &U);
+        if (slots == 4 && !zreg) kern = pick_keystream_kernel<C, LAYOUT, 4, false>(h, &U);
+        if (slots == 8 && !zreg) kern = pick_keystream_kernel<C, LAYOUT, 8, false>(h, &U);
+    }
     bsk::KsArgs a{};
     a.state = h->state;
     a.Gp = h->Gp;
@@ -216,7 +273,8 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
     const bool ws_pref = h->opt_rm_ws < 0 ? (C::U_DEFAULT != 32) : (h->opt_rm_ws != 0);
     const bool ws = LAYOUT == bsk::L_ROW_MAJOR && ws_pref && h->opt_sched != 0;
     int block = KS_BLOCK, compute_warps = KS_BLOCK / 32;
-    size_t smem = LAYOUT == bsk::L_ROW_MAJOR ? size_t(KS_BLOCK / 32) * bsk::RM_WARP_WORDS * 4 : 0;
+    size_t smem = LAYOUT == bsk::L_ROW_MAJOR ? size_t(KS_BLOCK / 32) * bsk::rm_warp_words(U, slots, zreg) * 4 : 0;
+    if (tmem) smem = (U == 32 && zreg) ? 0 : size_t(KS_BLOCK / 32) * bsk::ZS_WORDS * 4;
     if (ws) {
         kern = &bsk::keystream_rm_ws_kernel<C, C::U_DEFAULT>;
         if (h->opt_unroll == C::U_ALT0) kern = &bsk::keystream_rm_ws_kernel<C, C::U_ALT0>;
@@ -230,6 +288,7 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
         if (e != cudaSuccess) return fail(BSRNG_ECUDA, "smem attribute: %s", cudaGetErrorString(e));
     }
     unsigned grid;
+    int dbg_occ = 0, dbg_occ_max = 0;
     if (h->opt_sched == 0) {
         a.persistent = 0;
         a.nseg = 1;
@@ -252,7 +311,11 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
             whole_units = !ws && occ_max >= 2 && h->units >= 3 * slots2;
             occ = whole_units ? 2 : 1;
         }
-        if (occ > occ_max) occ = occ_max;
+        // an explicit setting is honoured even above the occupancy API's
+        // estimate (extra CTAs queue; the ticket order cannot deadlock)
+        if (occ > occ_max && h->opt_ctas_per_sm <= 0) occ = occ_max;
+        dbg_occ = occ;
+        dbg_occ_max = occ_max;
         const uint64_t slots = uint64_t(h->num_sms) * occ * compute_warps;  // resident clock-loop warps
         uint64_t nseg = 1;
         if (h->opt_seg_clocks) {
@@ -295,7 +358,8 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
         unsigned long long c[4];
         cudaMemcpyAsync(c, dbg, sizeof c, cudaMemcpyDeviceToHost, st);
         cudaStreamSynchronize(st);
-        fprintf(stderr, "[bsrng] grid=%u units=%llu nseg=%llu seg=%llu: waits=%llu slept=%llu spins=%llu\n", grid,
+        fprintf(stderr, "[bsrng] occ=%d/%d smem=%zu grid=%u units=%llu nseg=%llu seg=%llu: waits=%llu slept=%llu spins=%llu\n",
+                dbg_occ, dbg_occ_max, smem, grid,
                 (unsigned long long)a.units, (unsigned long long)a.nseg, (unsigned long long)a.seg_clocks, c[0], c[1],
                 c[2]);
         cudaFree(dbg);
@@ -373,7 +437,7 @@ int launch_aes_rowmajor_lanes(bsrng_t* h, void* out, uint64_t bits, cudaStream_t
     a.out = out;
     a.row_bytes = bits / 8;
     a.units = h->G;  // one warp = 32 instances
-    a.aux = h->raw + h->key_rows * h->key_bytes;
+    a.aux = h->raw + h->iv_off;
     a.persistent = 1;
     a.ticket = h->sched;
     a.flags = h->sched + 1;
@@ -487,11 +551,16 @@ bsrng_t* bsrng_create_ex(bsrng_cipher cipher, const uint8_t* keys, const uint8_t
     h->key_bytes = (aes || lfsr) ? 16 : 10;
     h->iv_bytes = cipher == BSRNG_GRAIN_V1 ? 8 : aes ? 16 : lfsr ? 0 : 10;
     h->key_rows = aes ? 1 : h->n;
+    // the fused init kernels (MICKEY, Grain) read whole 32-instance group
+    // blocks with 16 B loads: both regions padded to Gp*32 rows and zeroed
+    const bool padded = cipher == BSRNG_MICKEY2 || cipher == BSRNG_GRAIN_V1;
+    h->iv_off = padded ? h->Gp * 32 * h->key_bytes : h->key_rows * h->key_bytes;
+    const uint64_t raw_bytes = h->iv_off + (padded ? h->Gp * 32 : h->n) * h->iv_bytes;
     const int ns = nstate_of(cipher);
     const uint64_t sl_words = (aes || lfsr) ? 1 : uint64_t(h->key_bytes + h->iv_bytes) * 8 * h->Gp;
     if (cudaMalloc(&h->state, uint64_t(ns + 1) * h->Gp * 4) != cudaSuccess ||
         cudaMalloc(&h->sliced, sl_words * 4) != cudaSuccess ||
-        cudaMalloc(&h->raw, h->key_rows * h->key_bytes + h->n * h->iv_bytes) != cudaSuccess ||
+        cudaMalloc(&h->raw, raw_bytes) != cudaSuccess ||
         cudaMalloc(&h->sched, (1 + h->units + 32) * 4) != cudaSuccess ||
         (aes && cudaMalloc(&h->rk_dev, sizeof(bsk::aes::RoundKeys)) != cudaSuccess)) {
         cudaGetLastError();
@@ -500,6 +569,11 @@ bsrng_t* bsrng_create_ex(bsrng_cipher cipher, const uint8_t* keys, const uint8_t
         return nullptr;
     }
     cudaStream_t st = static_cast<cudaStream_t>(stream);
+    if (padded && cudaMemsetAsync(h->raw, 0, raw_bytes, st) != cudaSuccess) {
+        bsrng_destroy(h);
+        fail(BSRNG_ECUDA, "memset(raw) failed");
+        return nullptr;
+    }
     if (bsrng_rekey(h, keys, ivs, flags, stream) != BSRNG_OK) {
         std::string msg = g_err;
         bsrng_destroy(h);
@@ -530,7 +604,7 @@ int bsrng_rekey(bsrng_t* h, const uint8_t* keys, const uint8_t* ivs, uint32_t fl
     if (!dg.ok) return fail(BSRNG_ECUDA, "cudaSetDevice(%d) failed", h->dev);
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     if (!ivs) {  // iv_bits == 0: IV bytes are never read; keep them defined
-        cudaError_t e = cudaMemsetAsync(h->raw + h->key_rows * h->key_bytes, 0, h->n * h->iv_bytes, st);
+        cudaError_t e = cudaMemsetAsync(h->raw + h->iv_off, 0, h->n * h->iv_bytes, st);
         if (e != cudaSuccess) return fail(BSRNG_ECUDA, "memset: %s", cudaGetErrorString(e));
         const cudaMemcpyKind kind = (flags & BSRNG_INPUT_DEVICE) ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
         e = cudaMemcpyAsync(h->raw, keys, h->key_rows * h->key_bytes, kind, st);
@@ -662,6 +736,18 @@ int bsrng_set_option(bsrng_t* h, const char* key, int64_t value)
     } else if (!strcmp(key, "rm_ws")) {
         if (value < -1 || value > 1) return fail(BSRNG_EINVAL, "rm_ws must be -1 (auto), 0 or 1");
         h->opt_rm_ws = int(value);
+    } else if (!strcmp(key, "rm_slots")) {
+        if (value != 0 && value != 4 && value != 8) return fail(BSRNG_EINVAL, "rm_slots must be 0 (auto), 4 or 8");
+        h->opt_rm_slots = int(value);
+    } else if (!strcmp(key, "rm_zreg")) {
+        if (value != 0 && value != 1) return fail(BSRNG_EINVAL, "rm_zreg must be 0 or 1");
+        h->opt_rm_zreg = int(value);
+    } else if (!strcmp(key, "rm_tmem")) {
+        if (value != 0 && value != 1) return fail(BSRNG_EINVAL, "rm_tmem must be 0 or 1");
+        h->opt_rm_tmem = int(value);
+    } else if (!strcmp(key, "init_fused")) {
+        if (value != 0 && value != 1) return fail(BSRNG_EINVAL, "init_fused must be 0 or 1");
+        h->opt_init_fused = int(value);
     } else if (!strcmp(key, "block")) {
         if (value != KS_BLOCK) return fail(BSRNG_EINVAL, "block=%lld not built (built: %d)", (long long)value, KS_BLOCK);
     } else {

@@ -73,21 +73,30 @@ __device__ __forceinline__ uint32_t lane_mask(const KsArgs& a, uint64_t g)
 }
 
 // ROW_MAJOR staging per warp (dynamic shared memory):
-//   zs: z words of the current 32-clock block, [t][lane]      (4 KB / warp)
-//   os: transposed words for one 32-byte sector of every row,
-//       [row q][slot k][lane], k = 32-clock block within the sector (32 KB)
+//   zs: z words of the current 32-clock block, [t][lane]      (4 KB / warp;
+//       not used when the cipher loop keeps the block in registers, U = 32)
+//   os: transposed words for one row segment of every row,
+//       [row q][slot k][lane], k = 32-clock block within the segment
+//       (SLOTS x 4 KB: SLOTS = 8 -> one whole 32 B DRAM sector per row,
+//       SLOTS = 4 -> half a sector, half the smem, so two CTAs fit per SM)
 // Every access is lane-contiguous, so STS/LDS are bank-conflict free.  Rows are
-// written as whole 32 B sectors (two 16 B stores): 4-byte stores spread over
-// the ~600k rows in flight overflowed L2 before their sectors filled, and the
-// partial-sector evictions cost ~15x the algorithmic DRAM traffic (ncu).
+// written as whole 16 B pieces: 4-byte stores spread over the ~600k rows in
+// flight overflowed L2 before their sectors filled, and the partial-sector
+// evictions cost ~15x the algorithmic DRAM traffic (ncu).
 constexpr int ZS_WORDS = 32 * 32;
-constexpr int OS_WORDS = 32 * 8 * 32;
+constexpr int OS_WORDS = 32 * 8 * 32;  // SLOTS = 8
 constexpr int RM_WARP_WORDS = ZS_WORDS + OS_WORDS;
+__host__ __device__ constexpr int os_words(int slots) { return 32 * slots * 32; }
+// zreg: the loop keeps its 32-clock z block in registers (U = 32 only)
+__host__ __device__ constexpr int rm_warp_words(int U, int slots, bool zreg)
+{
+    return (U == 32 && zreg ? 0 : ZS_WORDS) + os_words(slots);
+}
 
 // Transpose this thread's 32 staged z words (a 32x32 bit block) and park the
 // 32 row words in sector slot `k`.  Bit-matrix row t is clock t, or clock t^7
 // for MSB-first ciphers so that clock 8b+q lands in bit 7-q of byte b.
-template <bool MSB_FIRST>
+template <bool MSB_FIRST, int SLOTS = 8>
 __device__ __forceinline__ void rowmajor_transpose(const uint32_t* zs, uint32_t* os, uint32_t k)
 {
     constexpr int X = MSB_FIRST ? 7 : 0;
@@ -102,12 +111,12 @@ __device__ __forceinline__ void rowmajor_transpose(const uint32_t* zs, uint32_t*
         }
         bt_transpose16(x);
 #pragma unroll
-        for (int q = 0; q < 16; ++q) os[((16 * h + q) * 8 + k) * 32] = x[q];
+        for (int q = 0; q < 16; ++q) os[((16 * h + q) * SLOTS + k) * 32] = x[q];
     }
 }
 
 // The same from 32 z words held in registers (cipher loops unrolled 32x).
-template <bool MSB_FIRST>
+template <bool MSB_FIRST, int SLOTS = 8>
 __device__ __forceinline__ void rowmajor_transpose_regs(const uint32_t (&z)[32], uint32_t* os, uint32_t k)
 {
     constexpr int X = MSB_FIRST ? 7 : 0;
@@ -118,61 +127,214 @@ __device__ __forceinline__ void rowmajor_transpose_regs(const uint32_t (&z)[32],
         for (int q = 0; q < 16; ++q) x[q] = __byte_perm(z[q ^ X], z[(q + 16) ^ X], h == 0 ? 0x5410 : 0x7632);
         bt_transpose16(x);
 #pragma unroll
-        for (int q = 0; q < 16; ++q) os[((16 * h + q) * 8 + k) * 32] = x[q];
+        for (int q = 0; q < 16; ++q) os[((16 * h + q) * SLOTS + k) * 32] = x[q];
     }
+}
+
+// 16 B row store: whole-sector flushes (SLOTS = 8) stream past L2
+// (evict-first); half-sector flushes (SLOTS = 4) keep normal L2 priority so
+// the sector's first half is still resident when its second half arrives.
+template <int SLOTS>
+__device__ __forceinline__ void st_row16(uint4* d, uint4 v)
+{
+    if constexpr (SLOTS == 8)
+        __stcs(d, v);
+    else
+        __stcg(d, v);
 }
 
 // Write slots [k_lo, k_hi] of every real row of this thread's group.
 //   row0: address of instance 32g's row; col: byte column of slot k_lo.
-// Full sectors go out as two 16 B stores (or four 8 B stores when rows are only
-// 8 B aligned, e.g. the paper's 4416-clock rows of 552 B); partial sectors at
+// Full segments go out as SLOTS/4 16 B stores (or 8 B stores when rows are only
+// 8 B aligned, e.g. the paper's 4416-clock rows of 552 B); partial segments at
 // item boundaries word by word.
+template <int SLOTS = 8>
 __device__ __forceinline__ void rowmajor_store(const uint32_t* os, uint8_t* row0, uint64_t row_bytes,
                                                uint32_t nvalid, uint32_t k_lo, uint32_t k_hi, uint64_t col)
 {
+    static_assert(SLOTS == 4 || SLOTS == 8, "SLOTS must be 4 or 8");
     uint8_t* p = row0 + col;
     const uint64_t align = reinterpret_cast<uintptr_t>(p) | row_bytes;
-    if (k_lo == 0 && k_hi == 7 && (align & 15) == 0 && nvalid == 32) {
-        // all shared-memory loads of 8 rows first, then their 16 stores, so a
+    if (k_lo == 0 && k_hi == SLOTS - 1 && (align & 15) == 0 && nvalid == 32) {
+        // all shared-memory loads of 8 rows first, then their stores, so a
         // lone warp does not wait out each load -> store latency per row
 #pragma unroll 1
         for (uint32_t q0 = 0; q0 < 32; q0 += 8) {
-            uint32_t v[8][8];
+            uint32_t v[8][SLOTS];
 #pragma unroll
             for (int r = 0; r < 8; ++r)
 #pragma unroll
-                for (int k = 0; k < 8; ++k) v[r][k] = os[((q0 + r) * 8 + k) * 32];
+                for (int k = 0; k < SLOTS; ++k) v[r][k] = os[((q0 + r) * SLOTS + k) * 32];
 #pragma unroll
             for (int r = 0; r < 8; ++r) {
                 uint4* d = reinterpret_cast<uint4*>(p + (q0 + r) * row_bytes);
-                __stcs(d, make_uint4(v[r][0], v[r][1], v[r][2], v[r][3]));
-                __stcs(d + 1, make_uint4(v[r][4], v[r][5], v[r][6], v[r][7]));
+#pragma unroll
+                for (int k = 0; k < SLOTS; k += 4)
+                    st_row16<SLOTS>(d + k / 4, make_uint4(v[r][k], v[r][k + 1], v[r][k + 2], v[r][k + 3]));
             }
         }
-    } else if (k_lo == 0 && k_hi == 7 && (align & 15) == 0) {
+    } else if (k_lo == 0 && k_hi == SLOTS - 1 && (align & 15) == 0) {
 #pragma unroll 4
         for (uint32_t q = 0; q < nvalid; ++q) {
-            const uint32_t* src = os + q * 8 * 32;
-            const uint4 v0 = make_uint4(src[0], src[32], src[64], src[96]);
-            const uint4 v1 = make_uint4(src[128], src[160], src[192], src[224]);
+            const uint32_t* src = os + q * SLOTS * 32;
             uint4* d = reinterpret_cast<uint4*>(p + q * row_bytes);
-            __stcs(d, v0);
-            __stcs(d + 1, v1);
+#pragma unroll
+            for (int k = 0; k < SLOTS; k += 4)
+                st_row16<SLOTS>(d + k / 4, make_uint4(src[k * 32], src[(k + 1) * 32], src[(k + 2) * 32],
+                                                      src[(k + 3) * 32]));
         }
-    } else if (k_lo == 0 && k_hi == 7 && (align & 7) == 0) {
+    } else if (k_lo == 0 && k_hi == SLOTS - 1 && (align & 7) == 0) {
 #pragma unroll 4
         for (uint32_t q = 0; q < nvalid; ++q) {
-            const uint32_t* src = os + q * 8 * 32;
+            const uint32_t* src = os + q * SLOTS * 32;
             uint2* d = reinterpret_cast<uint2*>(p + q * row_bytes);
-            __stcs(d, make_uint2(src[0], src[32]));
-            __stcs(d + 1, make_uint2(src[64], src[96]));
-            __stcs(d + 2, make_uint2(src[128], src[160]));
-            __stcs(d + 3, make_uint2(src[192], src[224]));
+#pragma unroll
+            for (int k = 0; k < SLOTS; k += 2) __stcs(d + k / 2, make_uint2(src[k * 32], src[(k + 1) * 32]));
         }
     } else {
         for (uint32_t q = 0; q < nvalid; ++q)
             for (uint32_t k = k_lo; k <= k_hi; ++k)
-                __stcs(reinterpret_cast<uint32_t*>(p + q * row_bytes + (k - k_lo) * 4), os[(q * 8 + k) * 32]);
+                __stcs(reinterpret_cast<uint32_t*>(p + q * row_bytes + (k - k_lo) * 4), os[(q * SLOTS + k) * 32]);
+    }
+}
+
+// ---------------------------------------------------------------------------
+// ROW_MAJOR staging in tensor memory (sm_100a TMEM, 128 lanes x 512 columns x
+// 32 bit per SM).  Nothing here is a matrix product: TMEM is used as a plain
+// per-thread staging buffer, because the whole-sector row buffer (32 rows x 8
+// slots per thread = 32 KB per warp) does not fit twice per SMSP in shared
+// memory, and half-sector flushes make L2 fetch and re-evict sectors (ncu:
+// 13 GB of DRAM reads and 2x the writes for 8.6 GB of Grain keystream).  Warp
+// w of a 4-warp CTA owns TMEM lanes 32(w%4)..+31 (its lane quarter); thread t
+// stores row q's word for slot k at column k*32 + q of lane 32(w%4)+t.  Each
+// CTA allocates 256 columns, so two CTAs (two clock-loop warps per SMSP) fit.
+// ---------------------------------------------------------------------------
+constexpr uint32_t TMEM_COLS = 256;
+
+__device__ __forceinline__ uint32_t tmem_alloc_cta(uint32_t* s_base)
+{
+    if ((threadIdx.x >> 5) == 0) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                         static_cast<uint32_t>(__cvta_generic_to_shared(s_base))),
+                     "n"(TMEM_COLS)
+                     : "memory");
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    return *reinterpret_cast<volatile uint32_t*>(s_base);
+}
+
+__device__ __forceinline__ void tmem_dealloc_cta(uint32_t base)
+{
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    if ((threadIdx.x >> 5) == 0)
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(base), "n"(TMEM_COLS) : "memory");
+}
+
+// 16 consecutive columns of this thread's lane <- x[0..15]
+__device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&x)[16])
+{
+    asm volatile(
+        "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, "
+        "%14, %15, %16};" ::"r"(taddr),
+        "r"(x[0]), "r"(x[1]), "r"(x[2]), "r"(x[3]), "r"(x[4]), "r"(x[5]), "r"(x[6]), "r"(x[7]), "r"(x[8]),
+        "r"(x[9]), "r"(x[10]), "r"(x[11]), "r"(x[12]), "r"(x[13]), "r"(x[14]), "r"(x[15])
+        : "memory");
+}
+
+// v[0..7] <- 8 consecutive columns of this thread's lane (load + wait in one
+// asm block, so no use of v can be scheduled before the data has arrived)
+__device__ __forceinline__ void tmem_ld8(uint32_t taddr, uint32_t (&v)[8])
+{
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];\n\t"
+        "tcgen05.wait::ld.sync.aligned;"
+        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7])
+        : "r"(taddr)
+        : "memory");
+}
+
+__device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
+
+// Transpose 32 z words held in registers and park the row words of slot k in
+// TMEM columns k*32 + q (tm = this warp's lane-quarter base address).
+template <bool MSB_FIRST>
+__device__ __forceinline__ void rowmajor_transpose_tmem(const uint32_t (&z)[32], uint32_t tm, uint32_t k)
+{
+    constexpr int X = MSB_FIRST ? 7 : 0;
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+        uint32_t x[16];
+#pragma unroll
+        for (int q = 0; q < 16; ++q) x[q] = __byte_perm(z[q ^ X], z[(q + 16) ^ X], h == 0 ? 0x5410 : 0x7632);
+        bt_transpose16(x);
+        tmem_st16(tm + k * 32 + 16 * h, x);
+    }
+}
+// The same from 32 z words staged in shared memory ([t][lane], zs = lane's column).
+template <bool MSB_FIRST>
+__device__ __forceinline__ void rowmajor_transpose_smem_tmem(const uint32_t* zs, uint32_t tm, uint32_t k)
+{
+    constexpr int X = MSB_FIRST ? 7 : 0;
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+        uint32_t x[16];
+#pragma unroll
+        for (int q = 0; q < 16; ++q)
+            x[q] = __byte_perm(zs[(q ^ X) * 32], zs[((q + 16) ^ X) * 32], h == 0 ? 0x5410 : 0x7632);
+        bt_transpose16(x);
+        tmem_st16(tm + k * 32 + 16 * h, x);
+    }
+}
+
+// Flush slots [k_lo, k_hi] of every real row from TMEM (rowmajor_store's
+// contract).  The loads are warp-collective, so every lane runs all of them;
+// the per-lane row count only predicates the global stores.
+__device__ __forceinline__ void rowmajor_store_tmem(uint32_t tm, uint8_t* row0, uint64_t row_bytes, uint32_t nvalid,
+                                                    uint32_t k_lo, uint32_t k_hi, uint64_t col)
+{
+    tmem_wait_st();
+    uint8_t* p = row0 + col;
+    const uint64_t align = reinterpret_cast<uintptr_t>(p) | row_bytes;
+    const bool full = k_lo == 0 && k_hi == 7;
+#pragma unroll 1
+    for (uint32_t q0 = 0; q0 < 32; q0 += 8) {
+        uint32_t v[8][8];  // [slot][row]
+#pragma unroll
+        for (int k = 0; k < 8; ++k) tmem_ld8(tm + k * 32 + q0, v[k]);
+        if (full && (align & 15) == 0) {
+#pragma unroll
+            for (int r = 0; r < 8; ++r) {
+                if (q0 + r < nvalid) {
+                    uint4* d = reinterpret_cast<uint4*>(p + (q0 + r) * row_bytes);
+                    __stcs(d, make_uint4(v[0][r], v[1][r], v[2][r], v[3][r]));
+                    __stcs(d + 1, make_uint4(v[4][r], v[5][r], v[6][r], v[7][r]));
+                }
+            }
+        } else if (full && (align & 7) == 0) {
+#pragma unroll
+            for (int r = 0; r < 8; ++r) {
+                if (q0 + r < nvalid) {
+                    uint2* d = reinterpret_cast<uint2*>(p + (q0 + r) * row_bytes);
+#pragma unroll
+                    for (int k = 0; k < 8; k += 2) __stcs(d + k / 2, make_uint2(v[k][r], v[k + 1][r]));
+                }
+            }
+        } else {
+#pragma unroll
+            for (int r = 0; r < 8; ++r) {
+                if (q0 + r < nvalid) {
+                    uint32_t* d = reinterpret_cast<uint32_t*>(p + (q0 + r) * row_bytes);
+#pragma unroll
+                    for (int k = 0; k < 8; ++k)
+                        if (uint32_t(k) >= k_lo && uint32_t(k) <= k_hi) __stcs(d + (k - k_lo), v[k][r]);
+                }
+            }
+        }
     }
 }
 
@@ -191,12 +353,14 @@ __device__ __forceinline__ void next_item(const KsArgs& a, volatile uint32_t* sl
     __syncwarp();
 }
 
-template <class C, int LAYOUT, int U, int BLOCK>
+// SLOTS: row-segment slots staged in smem (8 or 4); TMEM: stage in tensor
+// memory instead (8 slots, no smem for rows); ZREG: see rm_warp_words.
+template <class C, int LAYOUT, int U, int BLOCK, int SLOTS = 8, bool ZREG = true, bool TMEM = false>
 __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
 {
     static_assert(32 % U == 0, "U must divide 32");
     constexpr int NW = BLOCK / 32;
-    extern __shared__ uint32_t rm_smem[];  // ROW_MAJOR only: NW * RM_WARP_WORDS
+    extern __shared__ uint32_t rm_smem[];  // ROW_MAJOR only: NW * rm_warp_words(U, SLOTS, ZREG) (none with TMEM and ZREG)
     __shared__ uint8_t* s_row0[LAYOUT == L_ROW_MAJOR ? BLOCK : 1];
     __shared__ uint32_t s_nvalid[LAYOUT == L_ROW_MAJOR ? BLOCK : 1];
     __shared__ uint32_t s_item[NW];
@@ -204,6 +368,17 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
     // other per-item value is re-derived afterwards, so the 200 state words
     // plus temporaries fit in 255 registers without spilling.
     volatile uint32_t* slot = s_item + (threadIdx.x >> 5);
+    // TMEM staging: the CTA's allocation base lives in smem and each use
+    // re-derives this warp's lane-quarter address (no register held across
+    // the clock loop)
+    __shared__ uint32_t s_tmem;
+    if constexpr (LAYOUT == L_ROW_MAJOR && TMEM) {
+        static_assert(BLOCK == 128, "TMEM staging maps warp w to lane quarter w");
+        (void)tmem_alloc_cta(&s_tmem);
+    }
+    auto tm_addr = [&]() {
+        return *reinterpret_cast<volatile uint32_t*>(&s_tmem) + ((threadIdx.x >> 5) << 21);
+    };
     if (a.persistent)
         next_item(a, slot);
     else if (laneid_volatile() == 0)
@@ -273,14 +448,16 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
             const uint32_t nvalid = first >= a.n ? 0u : uint32_t(a.n - first < 32 ? a.n - first : 32);
             s_row0[threadIdx.x] = static_cast<uint8_t*>(a.out) + (nvalid ? first : 0) * a.row_bytes;
             s_nvalid[threadIdx.x] = nvalid;
-            uint32_t* zs = rm_smem + (threadIdx.x >> 5) * RM_WARP_WORDS + lane;
+            uint32_t* zs = rm_smem + (threadIdx.x >> 5) * (TMEM ? ZS_WORDS : rm_warp_words(U, SLOTS, ZREG)) + lane;
+            uint32_t* os = zs + (U == 32 && ZREG ? 0 : ZS_WORDS);
             const uint64_t b0 = clk_begin >> 5;  // call-relative index of the first 32-clock block
             const uint32_t nblk = nclk >> 5;
+            constexpr uint32_t NSLOT = TMEM ? 8 : SLOTS;
 #pragma unroll 1
             for (uint32_t blk = 0; blk < nblk; ++blk) {
                 const uint64_t B = b0 + blk;
-                const uint32_t k = uint32_t(B & 7);
-                if constexpr (U == 32) {
+                const uint32_t k = uint32_t(B & (NSLOT - 1));
+                if constexpr (U == 32 && ZREG) {
                     // one 32-clock block per iteration: keep the z words in
                     // registers and transpose them there (no z staging in smem)
                     uint32_t zr[32];
@@ -289,7 +466,10 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
                         zr[u] = c.z();
                         c.clock();
                     }
-                    rowmajor_transpose_regs<C::MSB_FIRST>(zr, zs + ZS_WORDS, k);
+                    if constexpr (TMEM)
+                        rowmajor_transpose_tmem<C::MSB_FIRST>(zr, tm_addr(), k);
+                    else
+                        rowmajor_transpose_regs<C::MSB_FIRST, SLOTS>(zr, os, k);
                 } else {
 #pragma unroll 1
                     for (uint32_t kk = 0; kk < 32; kk += U) {
@@ -299,12 +479,19 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
                             c.clock();
                         }
                     }
-                    rowmajor_transpose<C::MSB_FIRST>(zs, zs + ZS_WORDS, k);
+                    if constexpr (TMEM)
+                        rowmajor_transpose_smem_tmem<C::MSB_FIRST>(zs, tm_addr(), k);
+                    else
+                        rowmajor_transpose<C::MSB_FIRST, SLOTS>(zs, os, k);
                 }
-                if (k == 7 || blk + 1 == nblk) {
+                if (k == NSLOT - 1 || blk + 1 == nblk) {
                     const uint32_t k_lo = k - (blk < k ? blk : k);
-                    rowmajor_store(zs + ZS_WORDS, s_row0[threadIdx.x], a.row_bytes, s_nvalid[threadIdx.x], k_lo,
-                                   k, (B - (k - k_lo)) * 4);
+                    if constexpr (TMEM)
+                        rowmajor_store_tmem(tm_addr(), s_row0[threadIdx.x], a.row_bytes, s_nvalid[threadIdx.x], k_lo, k,
+                                            (B - (k - k_lo)) * 4);
+                    else
+                        rowmajor_store<SLOTS>(os, s_row0[threadIdx.x], a.row_bytes, s_nvalid[threadIdx.x], k_lo, k,
+                                              (B - (k - k_lo)) * 4);
                 }
             }
         }
@@ -339,6 +526,7 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
         }
         next_item(a, slot);
     }
+    if constexpr (LAYOUT == L_ROW_MAJOR && TMEM) tmem_dealloc_cta(*reinterpret_cast<volatile uint32_t*>(&s_tmem));
 }
 
 }  // namespace bsk

@@ -159,16 +159,28 @@ __global__ void __launch_bounds__(128) m2_preclock_kernel(const uint32_t* __rest
 #pragma unroll
     for (int i = 0; i < 100; ++i) r[i] = s[i] = 0u;
     // 4 clocks per loop iteration (iv_bits is a multiple of 8): the S-register
-    // renaming then closes inside the body instead of costing ~100 moves/clock
-#pragma unroll 1
-    for (int i = 0; i < iv_bits; i += 4) {
+    // renaming then closes inside the body instead of costing ~100 moves/clock.
+    // The input words of the next 4 clocks are loaded one iteration ahead, so
+    // their HBM latency hides behind ~1300 LOP3 (ncu: long-scoreboard was the
+    // second stall reason without the prefetch).
+    const int nin = iv_bits + 80;
+    const uint32_t* iv_p = iv_s + g;
+    const uint32_t* key_p = key_s + g - uint64_t(iv_bits) * Gp;
+    auto in_ptr = [&](int c) { return (c < iv_bits ? iv_p : key_p) + uint64_t(c) * Gp; };
+    uint32_t cur[4];
 #pragma unroll
-        for (int u = 0; u < 4; ++u) m2::clock_kg<true>(r, s, iv_s[uint64_t(i + u) * Gp + g]);
-    }
+    for (int u = 0; u < 4; ++u) cur[u] = __ldcs(in_ptr(u));
 #pragma unroll 1
-    for (int i = 0; i < 80; i += 4) {
+    for (int c = 0; c < nin; c += 4) {
+        uint32_t nxt[4] = {0u, 0u, 0u, 0u};
+        if (c + 4 < nin) {
 #pragma unroll
-        for (int u = 0; u < 4; ++u) m2::clock_kg<true>(r, s, key_s[uint64_t(i + u) * Gp + g]);
+            for (int u = 0; u < 4; ++u) nxt[u] = __ldcs(in_ptr(c + 4 + u));
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) m2::clock_kg<true>(r, s, cur[u]);
+#pragma unroll
+        for (int u = 0; u < 4; ++u) cur[u] = nxt[u];
     }
 #pragma unroll 1
     for (int i = 0; i < 100; i += 4) {
@@ -180,6 +192,64 @@ __global__ void __launch_bounds__(128) m2_preclock_kernel(const uint32_t* __rest
 #pragma unroll
     for (int i = 0; i < 100; ++i) state[uint64_t(100 + i) * Gp + g] = s[i];
     state[uint64_t(200) * Gp + g] = 0u;
+}
+
+}  // namespace bsk
+
+namespace bsk {
+
+// ---------------------------------------------------------------------------
+// Fused key/IV slicing + preclock (SURVEY steps a-1 + a-2 in one kernel).
+//
+// The separate path (slice_bits_kernel x2 -> sliced words in HBM ->
+// m2_preclock_kernel) spent ~20% of a rekey in the two slicing launches and
+// re-read every input word from HBM inside the clock loop.  Here each thread
+// (one group, as in the clock loop) loads its 32 instances' IV and key bytes
+// with 16 B loads, slices them in registers (slice_group32: PRMT + the 32x32
+// bit transpose) while the cipher state is still all-zero (no extra register
+// pressure), and parks the 160 slice words in shared memory [bit][thread];
+// the 260 mixing clocks then read their input word from shared memory.
+// 20 KB of smem per warp -> two 4-warp CTAs (two warps per SMSP) per SM.
+// Inputs: raw_k / raw_iv regions of Gp*32*10 bytes, 16 B aligned, zero
+// beyond instance n (bsrng.cu allocates and zero-fills them).
+// ---------------------------------------------------------------------------
+constexpr int M2I_BLOCK = 128;
+constexpr size_t M2I_SMEM_BYTES = size_t(160) * M2I_BLOCK * 4;  // [IV bit 0..79, key bit 0..79][thread]
+
+__global__ void __launch_bounds__(M2I_BLOCK, 2) m2_init_kernel(const uint8_t* __restrict__ raw_k,
+                                                              const uint8_t* __restrict__ raw_iv, int iv_bits,
+                                                              uint32_t* __restrict__ state, uint64_t Gp)
+{
+    extern __shared__ uint32_t m2i_smem[];
+    const uint64_t g = uint64_t(blockIdx.x) * M2I_BLOCK + threadIdx.x;
+    if (g >= Gp) return;  // no block-level barrier below
+    uint32_t* sl = m2i_smem + threadIdx.x;
+    slice_group32<10, 80, true>(raw_iv + g * 320u, [&](int bit, uint32_t w) { sl[bit * M2I_BLOCK] = w; });
+    slice_group32<10, 80, true>(raw_k + g * 320u, [&](int bit, uint32_t w) { sl[(80 + bit) * M2I_BLOCK] = w; });
+
+    uint32_t r[100], s[100];
+#pragma unroll
+    for (int i = 0; i < 100; ++i) r[i] = s[i] = 0u;
+    const int nin = iv_bits + 80;  // IV clocks, then key clocks: rows 0..iv_bits-1, 80..159
+#pragma unroll 1
+    for (int c = 0; c < nin; c += 4) {
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            const int row = c + u < iv_bits ? c + u : c + u - iv_bits + 80;
+            m2::clock_kg<true>(r, s, sl[row * M2I_BLOCK]);
+        }
+    }
+#pragma unroll 1
+    for (int i = 0; i < 100; i += 4) {
+#pragma unroll
+        for (int u = 0; u < 4; ++u) m2::clock_kg<true>(r, s, 0u);
+    }
+    uint32_t* p = opaque(state + g);
+#pragma unroll
+    for (int i = 0; i < 100; ++i) __stcg(p + uint64_t(i) * Gp, r[i]);
+#pragma unroll
+    for (int i = 0; i < 100; ++i) __stcg(p + uint64_t(100 + i) * Gp, s[i]);
+    p[uint64_t(200) * Gp] = 0u;
 }
 
 }  // namespace bsk

@@ -53,6 +53,9 @@ def test_zero_bits_is_noop(cipher):
     ("mickey2", {"ctas_per_sm": 2}), ("mickey2", {"rm_ws": 0}), ("mickey2", {"rm_ws": 1, "seg_clocks": 512}),
     ("grain", {"unroll": 8}), ("grain", {"unroll": 16}), ("grain", {"rm_ws": 1}), ("grain", {"sched": 0}),
     ("grain", {"ctas_per_sm": 1, "seg_clocks": 256}),
+    ("grain", {"rm_slots": 8}), ("grain", {"rm_slots": 4, "rm_zreg": 0}), ("grain", {"rm_slots": 8, "rm_zreg": 0}),
+    ("grain", {"rm_slots": 4, "ctas_per_sm": 2, "seg_clocks": 384}),
+    ("mickey2", {"rm_ws": 0, "rm_slots": 4}), ("mickey2", {"rm_ws": 0, "rm_slots": 4, "seg_clocks": 160}),
     ("aes128ctr", {"ctas_per_sm": 1}), ("aes128ctr", {"rm_ws": 0}), ("aes128ctr", {"seg_clocks": 4096}),
 ])
 def test_options_stay_bit_exact(cipher, opts):
@@ -76,7 +79,8 @@ def test_options_stay_bit_exact(cipher, opts):
 def test_option_validation():
     keys, ivs = inputs.make_inputs("grain", 32)
     g = bsrng.Generator("grain", keys, ivs)
-    for k, v in (("unroll", 4), ("sched", 2), ("seg_clocks", 33), ("ctas_per_sm", 99), ("rm_ws", 5)):
+    for k, v in (("unroll", 4), ("sched", 2), ("seg_clocks", 33), ("ctas_per_sm", 99), ("rm_ws", 5),
+                 ("rm_slots", 2), ("rm_zreg", 3), ("rm_tmem", 2)):
         with pytest.raises(bsrng.BsrngError) as e:
             g.set_option(k, v)
         assert e.value.code == bsrng.EINVAL
@@ -124,3 +128,31 @@ def test_mickey_2_40_limit_boundary():
         g.generate(buf, (1 << 40) + 32, "checksum")
     assert e.value.code == bsrng.ERANGE
     assert g.bits_done == 0
+
+
+@pytest.mark.parametrize("cipher,opts,bits", [
+    ("grain", {"rm_tmem": 1}, 8192),
+    ("grain", {"rm_tmem": 1}, 4416),                      # 552 B rows: 8 B-aligned flushes
+    ("grain", {"rm_tmem": 1, "seg_clocks": 160}, 2080),   # partial slots at segment ends
+    ("grain", {"rm_tmem": 1, "rm_zreg": 0}, 8192),
+    ("grain", {"rm_tmem": 1, "unroll": 16}, 4128),
+    ("grain", {"rm_tmem": 1, "sched": 0}, 2048),
+    ("grain", {"rm_tmem": 1, "ctas_per_sm": 2, "seg_clocks": 512}, 4096),
+    ("mickey2", {"rm_ws": 0, "rm_tmem": 1}, 4416),
+    ("mickey2", {"rm_ws": 0, "rm_tmem": 1, "seg_clocks": 96}, 1024),
+])
+def test_rm_tmem_staging_bit_exact(cipher, opts, bits):
+    """ROW_MAJOR with the row segments staged in tensor memory (TMEM) instead
+    of shared memory: every flush path (16 B, 8 B, partial words) bit-exact."""
+    n = 32 * 40 + 9
+    keys, ivs = inputs.make_inputs(cipher, n)
+    want = _want(cipher, keys, ivs, bits)
+    g = _gen(cipher, keys, ivs)
+    for k, v in opts.items():
+        g.set_option(k, v)
+    got = g.generate_host(bits, "row_major")
+    assert np.array_equal(got, want)
+    # a second call continues the streams (state carried through the handle)
+    got2 = g.generate_host(256, "row_major")
+    want2 = _want(cipher, keys, ivs, bits + 256)[:, bits // 8:]
+    assert np.array_equal(got2, want2)

@@ -53,12 +53,19 @@ def test_ragged_all_layouts(unroll):
             assert int(got[0]) == checksum(to_sliced(want, msb_first=False))
 
 
-def test_preclock_state_parity():
-    n = 70
+@pytest.mark.parametrize("init_fused", [1, 0])
+@pytest.mark.parametrize("n", [70, 1, 32 * 37 + 13])
+def test_preclock_state_parity(n, init_fused):
+    """a-1 + a-2 through the fused slicing + init kernel (default) and the
+    separate slice / init kernels (rekey re-runs the chosen path)."""
+    keys0, ivs0 = inputs.make_inputs("grain", n, seed=3)
+    g = bsrng.Generator("grain", keys0, ivs0)
+    g.set_option("init_fused", init_fused)
     keys, ivs = inputs.make_inputs("grain", n)
-    g = bsrng.Generator("grain", keys, ivs)
+    g.rekey(keys, ivs)
     real = np.full(g.groups, 0xFFFFFFFF, dtype=np.uint32)
-    real[-1] = (1 << (n - 32 * (g.groups - 1))) - 1
+    if n % 32:
+        real[-1] = (1 << (n % 32)) - 1
     for clocks in (0, 160):
         if clocks:
             g.generate_host(clocks, "checksum")

@@ -76,6 +76,34 @@ def test_preclock_state_parity():
         assert np.array_equal(g.copy_state() & real, want)
 
 
+@pytest.mark.parametrize("init_fused", [1, 0])
+@pytest.mark.parametrize("n,iv_bits", [(70, 80), (32 * 37 + 13, 80), (1, 80), (33, 0), (100, 24), (4096 + 5, 72)])
+def test_init_paths_state_parity(n, iv_bits, init_fused):
+    """a-1 + a-2: the fused slicing + preclock kernel (default) and the
+    separate slice / preclock kernels give the oracle's post-init state for
+    every real instance, at ragged n and short IVs; rekey uses the same path."""
+    keys, ivs = inputs.make_inputs("mickey2", n, seed=11)
+    g = bsrng.Generator("mickey2", keys, ivs, iv_bits=iv_bits)
+    g.set_option("init_fused", init_fused)
+    k2, v2 = inputs.make_inputs("mickey2", n, seed=12)
+    g.rekey(k2, v2)
+    real = np.full(g.groups, 0xFFFFFFFF, dtype=np.uint32)
+    if n % 32:
+        real[-1] = (1 << (n % 32)) - 1
+    idx = range(n) if n <= 256 else list(range(64)) + list(range(n - 64, n))
+    rs = {i: oracle.mickey2_state(bytes(k2[i]), bytes(v2[i]), iv_bits, 0) for i in idx}
+    st = g.copy_state()
+    for i in idx:
+        gi, j = divmod(i, 32)
+        got_r = (st[:100, gi] >> np.uint32(j)) & 1
+        got_s = (st[100:, gi] >> np.uint32(j)) & 1
+        assert np.array_equal(got_r, np.asarray(rs[i][0], dtype=np.uint32)), i
+        assert np.array_equal(got_s, np.asarray(rs[i][1], dtype=np.uint32)), i
+    # and the keystream that follows
+    want = oracle.mickey2_keystream_batch(k2[:40], v2[:40], iv_bits, 256)
+    assert np.array_equal(g.generate_host(256, "row_major")[:40], want)
+
+
 @pytest.mark.parametrize("iv_bits", [0, 32, 72])
 def test_short_ivs(iv_bits):
     n, bits = 40, 512

@@ -26,6 +26,7 @@ def main():
     p.add_argument("--seg-clocks", type=int, default=None)
     p.add_argument("--rm-ws", type=int, default=None)
     p.add_argument("--unroll", type=int, default=None)
+    p.add_argument("--opt", action="append", default=[], help="extra handle option key=value")
     a = p.parse_args()
     g = bsrng.Generator.from_seed(a.cipher, a.n)
     if a.sched is not None:
@@ -36,6 +37,9 @@ def main():
         g.set_option("rm_ws", a.rm_ws)
     if a.unroll is not None:
         g.set_option("unroll", a.unroll)
+    for kv in a.opt:
+        k, v = kv.split("=")
+        g.set_option(k, int(v))
     out = torch.empty(max(g.out_bytes(a.bits, a.layout), 16), dtype=torch.uint8, device="cuda")
     for _ in range(a.reps):
         g.generate(out, a.bits, a.layout)
