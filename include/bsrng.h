@@ -172,8 +172,9 @@ int64_t bsrng_copy_state(const bsrng_t* h, uint32_t* host_out, uint64_t words);
  *                  the z block in registers (1, default) or stage it in
  *                  shared memory (0)
  *   "rm_tmem"    : ROW_MAJOR plain kernel: stage the row segments in tensor
- *                  memory (TMEM, 256 columns per CTA) instead of shared
- *                  memory (1); default 0 (measured slower)
+ *                  memory (TMEM, 256 columns per CTA, two CTAs per SM) (1)
+ *                  or in shared memory (0); -1 = cipher default (Grain 1,
+ *                  MICKEY / LFSR 0)
  *   "init_fused" : MICKEY / Grain create/rekey: slicing fused into the
  *                  initialisation kernel (1, default) or the separate
  *                  slice_bits + preclock kernels (0)

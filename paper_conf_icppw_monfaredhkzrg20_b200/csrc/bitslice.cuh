@@ -191,6 +191,19 @@ __device__ __forceinline__ void slice_group32(const uint8_t* __restrict__ p, Put
     }
 }
 
+// Slice 32-instance group blocks straight into state rows [bit][Gp] (AES-CTR
+// initial counters, LFSR keys: the sliced input IS the state).  One thread
+// per group; raw = Gp*32 rows of NBYTES, 16 B aligned, zero past n.
+template <int NBYTES, int NBITS, bool MSB>
+__global__ void __launch_bounds__(128) slice_state_kernel(const uint8_t* __restrict__ raw,
+                                                          uint32_t* __restrict__ state, uint64_t Gp)
+{
+    const uint64_t g = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (g >= Gp) return;
+    uint32_t* p = state + g;
+    slice_group32<NBYTES, NBITS, MSB>(raw + g * (32u * NBYTES), [&](int bit, uint32_t w) { p[uint64_t(bit) * Gp] = w; });
+}
+
 // Hide a pointer's provenance from the optimiser (no code emitted beyond a
 // register move), so address arithmetic is not hoisted/CSE'd across the
 // register-resident clock loop.

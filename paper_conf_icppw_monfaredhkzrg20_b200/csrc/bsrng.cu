@@ -80,7 +80,7 @@ struct bsrng {
     uint32_t* state = nullptr;   // [NSTATE + 1][Gp]
     uint32_t* sliced = nullptr;  // key [KB][Gp] then iv [IVB][Gp]
     uint8_t* raw = nullptr;      // keys [n][key_bytes] then ivs [n][iv_bytes] at raw + iv_off
-    uint64_t iv_off = 0;         // MICKEY: both regions padded to Gp*32*10 B (zeroed), 16 B aligned
+    uint64_t iv_off = 0;         // per-instance regions padded to Gp*32 rows (zeroed), 16 B aligned
     uint32_t* sched = nullptr;   // [1 + units]: ticket, flags; then [32] scratch
     uint8_t* bounce = nullptr;   // generate_host staging
     uint32_t* rk_dev = nullptr;  // AES: round-key masks written by the key-expansion kernel
@@ -101,8 +101,9 @@ struct bsrng {
     // ROW_MAJOR, U = 32: z block in registers (1) or staged in smem (0).
     int opt_rm_zreg = 1;
     // ROW_MAJOR plain kernel: stage row segments in TMEM (1) or smem (0).
-    int opt_rm_tmem = 0;
-    // MICKEY / Grain init: fused slicing + preclock kernel (1) or slice kernels + preclock (0).
+    int opt_rm_tmem = -1;  // -1 = the cipher's default (C::RM_TMEM)
+    // init: slicing fused into the init kernel (MICKEY, Grain) / per-thread group
+    // slicing into the state (AES, LFSR) (1), or the ballot slice kernels (0).
     int opt_init_fused = 1;
 };
 
@@ -180,7 +181,10 @@ int run_init(bsrng_t* h, cudaStream_t st)
     case BSRNG_AES128_CTR: {
         // initial counter blocks sliced straight into the state rows (FIPS-197
         // bit order: bit 0 = MSB of byte 0); round keys from the one key.
-        bsk::slice_bits_kernel<16, 128, true><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_iv, h->n, h->state, h->Gp);
+        if (h->opt_init_fused)
+            bsk::slice_state_kernel<16, 128, true><<<unsigned((h->Gp + 127) / 128), 128, 0, st>>>(raw_iv, h->state, h->Gp);
+        else
+            bsk::slice_bits_kernel<16, 128, true><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_iv, h->n, h->state, h->Gp);
         if (int rc = check_launch("slice(ctr)")) return rc;
         bsk::aes::aes_key_expand_kernel<<<1, 32, 0, st>>>(raw_k, h->rk_dev);
         if (int rc = check_launch("aes_key_expand")) return rc;
@@ -195,7 +199,10 @@ int run_init(bsrng_t* h, cudaStream_t st)
     }
     case BSRNG_LFSR128: {
         // the state IS the key: 128 bits, MSB-first, sliced straight into rows 0..127
-        bsk::slice_bits_kernel<16, 128, true><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_k, h->n, h->state, h->Gp);
+        if (h->opt_init_fused)
+            bsk::slice_state_kernel<16, 128, true><<<unsigned((h->Gp + 127) / 128), 128, 0, st>>>(raw_k, h->state, h->Gp);
+        else
+            bsk::slice_bits_kernel<16, 128, true><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_k, h->n, h->state, h->Gp);
         if (int rc = check_launch("slice(key)")) return rc;
         cudaError_t e = cudaMemsetAsync(h->state + uint64_t(bsk::Lfsr128::NSTATE) * h->Gp, 0, h->Gp * 4, st);
         if (e != cudaSuccess) return fail(BSRNG_ECUDA, "memset: %s", cudaGetErrorString(e));
@@ -241,8 +248,13 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
     // U = 32 loops keep the 32-clock z block in registers (zreg) or stage it
     // in shared memory one word per clock (fewer live registers).
     const bool zreg = LAYOUT != bsk::L_ROW_MAJOR || h->opt_rm_zreg != 0;
-    // TMEM: stage the row segments in tensor memory instead of shared memory
-    const bool tmem = LAYOUT == bsk::L_ROW_MAJOR && h->opt_rm_tmem > 0;
+    // ROW_MAJOR kernel: warp-specialised compute/writer kernel (rowmajor_ws.cuh,
+    // 8 warps per CTA of which 4 run the clock loop; always persistent), or
+    // the plain clock kernel with the row segments staged in tensor memory
+    // (TMEM) or shared memory.  Defaults per cipher (RM_TMEM traits).
+    const bool ws_pref = h->opt_rm_ws < 0 ? (C::U_DEFAULT != 32 && !C::RM_TMEM) : (h->opt_rm_ws != 0);
+    const bool ws = LAYOUT == bsk::L_ROW_MAJOR && ws_pref && h->opt_sched != 0;
+    const bool tmem = LAYOUT == bsk::L_ROW_MAJOR && !ws && (h->opt_rm_tmem < 0 ? C::RM_TMEM : h->opt_rm_tmem > 0);
     int U = 0;
     auto kern = pick_keystream_kernel<C, LAYOUT, 8>(h, &U);
     if (tmem) {
@@ -268,10 +280,6 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
     a.units = h->units;
     a.scratch = h->sched + 1 + h->units;
 
-    // ROW_MAJOR default: warp-specialised compute/writer kernel (rowmajor_ws.cuh),
-    // 8 warps per CTA of which 4 run the clock loop; always persistent.
-    const bool ws_pref = h->opt_rm_ws < 0 ? (C::U_DEFAULT != 32) : (h->opt_rm_ws != 0);
-    const bool ws = LAYOUT == bsk::L_ROW_MAJOR && ws_pref && h->opt_sched != 0;
     int block = KS_BLOCK, compute_warps = KS_BLOCK / 32;
     size_t smem = LAYOUT == bsk::L_ROW_MAJOR ? size_t(KS_BLOCK / 32) * bsk::rm_warp_words(U, slots, zreg) * 4 : 0;
     if (tmem) smem = (U == 32 && zreg) ? 0 : size_t(KS_BLOCK / 32) * bsk::ZS_WORDS * 4;
@@ -299,6 +307,10 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_max, kern, block, smem) != cudaSuccess ||
             occ_max < 1)
             occ_max = 1;
+        // The occupancy API reports 1 CTA/SM for kernels that allocate tensor
+        // memory; registers (255 x 128 threads -> 2 CTAs) and TMEM (2 x 256 of
+        // 512 columns) allow two, which the GPU then runs (ncu: 7.9 warps/SM).
+        if (tmem) occ_max = 2;
         // Auto policy (opt_ctas_per_sm == 0).  Many more warp-units than warp
         // slots: two warps per SMSP, one item per unit (no time segments, so no
         // warp ever waits on another; a warp left alone at the end runs at
@@ -308,8 +320,8 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
         bool whole_units = false;
         if (occ <= 0) {
             const uint64_t slots2 = uint64_t(h->num_sms) * 2 * compute_warps;
-            whole_units = !ws && occ_max >= 2 && h->units >= 3 * slots2;
-            occ = whole_units ? 2 : 1;
+            whole_units = !ws && occ_max >= 2 && h->units >= 3 * slots2 && !(tmem && C::RM_SEGMENTED);
+            occ = (whole_units || tmem) ? 2 : 1;
         }
         // an explicit setting is honoured even above the occupancy API's
         // estimate (extra CTAs queue; the ticket order cannot deadlock)
@@ -323,7 +335,9 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
         } else if (!whole_units && h->units > slots) {
             // >= ~32 items per resident warp so the tail is <~3% of the call,
             // but segments no shorter than 256 clocks (state carry stays <1%)
-            nseg = std::max<uint64_t>(1, (32 * slots + h->units - 1) / h->units);
+            // (TMEM-staged ROW_MAJOR at two warps per SMSP: ~8 items per warp)
+            const uint64_t per_warp = tmem ? 8 : 32;
+            nseg = std::max<uint64_t>(1, (per_warp * slots + h->units - 1) / h->units);
             nseg = std::min<uint64_t>(nseg, std::max<uint64_t>(1, bits / 256));
         }
         // whole 256-clock blocks keep ROW_MAJOR sector flushes full (32 B/row)
@@ -551,11 +565,10 @@ bsrng_t* bsrng_create_ex(bsrng_cipher cipher, const uint8_t* keys, const uint8_t
     h->key_bytes = (aes || lfsr) ? 16 : 10;
     h->iv_bytes = cipher == BSRNG_GRAIN_V1 ? 8 : aes ? 16 : lfsr ? 0 : 10;
     h->key_rows = aes ? 1 : h->n;
-    // the fused init kernels (MICKEY, Grain) read whole 32-instance group
-    // blocks with 16 B loads: both regions padded to Gp*32 rows and zeroed
-    const bool padded = cipher == BSRNG_MICKEY2 || cipher == BSRNG_GRAIN_V1;
-    h->iv_off = padded ? h->Gp * 32 * h->key_bytes : h->key_rows * h->key_bytes;
-    const uint64_t raw_bytes = h->iv_off + (padded ? h->Gp * 32 : h->n) * h->iv_bytes;
+    // the fused init kernels read whole 32-instance group blocks with 16 B
+    // loads: the per-instance regions are padded to Gp*32 rows and zeroed
+    h->iv_off = aes ? 16 : h->Gp * 32 * h->key_bytes;  // AES: one 16 B key
+    const uint64_t raw_bytes = h->iv_off + h->Gp * 32 * h->iv_bytes;
     const int ns = nstate_of(cipher);
     const uint64_t sl_words = (aes || lfsr) ? 1 : uint64_t(h->key_bytes + h->iv_bytes) * 8 * h->Gp;
     if (cudaMalloc(&h->state, uint64_t(ns + 1) * h->Gp * 4) != cudaSuccess ||
@@ -569,7 +582,7 @@ bsrng_t* bsrng_create_ex(bsrng_cipher cipher, const uint8_t* keys, const uint8_t
         return nullptr;
     }
     cudaStream_t st = static_cast<cudaStream_t>(stream);
-    if (padded && cudaMemsetAsync(h->raw, 0, raw_bytes, st) != cudaSuccess) {
+    if (cudaMemsetAsync(h->raw, 0, raw_bytes, st) != cudaSuccess) {
         bsrng_destroy(h);
         fail(BSRNG_ECUDA, "memset(raw) failed");
         return nullptr;
@@ -743,7 +756,7 @@ int bsrng_set_option(bsrng_t* h, const char* key, int64_t value)
         if (value != 0 && value != 1) return fail(BSRNG_EINVAL, "rm_zreg must be 0 or 1");
         h->opt_rm_zreg = int(value);
     } else if (!strcmp(key, "rm_tmem")) {
-        if (value != 0 && value != 1) return fail(BSRNG_EINVAL, "rm_tmem must be 0 or 1");
+        if (value < -1 || value > 1) return fail(BSRNG_EINVAL, "rm_tmem must be -1 (auto), 0 or 1");
         h->opt_rm_tmem = int(value);
     } else if (!strcmp(key, "init_fused")) {
         if (value != 0 && value != 1) return fail(BSRNG_EINVAL, "init_fused must be 0 or 1");

@@ -119,6 +119,12 @@ struct Grain {
     // register rotation costs 160/U moves per clock at the back edge; at U = 32
     // ptxas emits them all as IMAD.MOV (FMA pipe), at U = 16 partly as MOV.
     static constexpr int U_DEFAULT = 32, U_ALT0 = 8, U_ALT1 = 16;
+    // ROW_MAJOR default: row segments staged in TMEM, two CTAs per SM (+7%
+    // over one CTA with smem staging; DESIGN.md sec. 5 Grain)
+    static constexpr bool RM_TMEM = true;
+    // ...with time segments (~8 per resident warp): a lone Grain warp keeps
+    // the ALU only ~70% busy, so a whole-unit tail wave would run slow
+    static constexpr bool RM_SEGMENTED = true;
     uint32_t s[80], b[80];
 
     __device__ __forceinline__ void load(const uint32_t* st, uint64_t Gp, uint64_t g)

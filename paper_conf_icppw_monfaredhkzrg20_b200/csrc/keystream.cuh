@@ -27,6 +27,7 @@
 //              32-bit word per instance row.
 #pragma once
 #include <cstdint>
+#include <utility>
 
 #include "bitslice.cuh"
 
@@ -156,17 +157,20 @@ __device__ __forceinline__ void rowmajor_store(const uint32_t* os, uint8_t* row0
     uint8_t* p = row0 + col;
     const uint64_t align = reinterpret_cast<uintptr_t>(p) | row_bytes;
     if (k_lo == 0 && k_hi == SLOTS - 1 && (align & 15) == 0 && nvalid == 32) {
-        // all shared-memory loads of 8 rows first, then their stores, so a
-        // lone warp does not wait out each load -> store latency per row
+        // all shared-memory loads of RB rows first, then their stores, so a
+        // lone warp does not wait out each load -> store latency per row.  The
+        // batch is 16 registers: more and ptxas spills MICKEY's state words
+        // inside the clock loop (it allocates the flush and the loop jointly)
+        constexpr int RB = 16 / SLOTS;
 #pragma unroll 1
-        for (uint32_t q0 = 0; q0 < 32; q0 += 8) {
-            uint32_t v[8][SLOTS];
+        for (uint32_t q0 = 0; q0 < 32; q0 += RB) {
+            uint32_t v[RB][SLOTS];
 #pragma unroll
-            for (int r = 0; r < 8; ++r)
+            for (int r = 0; r < RB; ++r)
 #pragma unroll
                 for (int k = 0; k < SLOTS; ++k) v[r][k] = os[((q0 + r) * SLOTS + k) * 32];
 #pragma unroll
-            for (int r = 0; r < 8; ++r) {
+            for (int r = 0; r < RB; ++r) {
                 uint4* d = reinterpret_cast<uint4*>(p + (q0 + r) * row_bytes);
 #pragma unroll
                 for (int k = 0; k < SLOTS; k += 4)
@@ -206,7 +210,8 @@ __device__ __forceinline__ void rowmajor_store(const uint32_t* os, uint8_t* row0
 // memory, and half-sector flushes make L2 fetch and re-evict sectors (ncu:
 // 13 GB of DRAM reads and 2x the writes for 8.6 GB of Grain keystream).  Warp
 // w of a 4-warp CTA owns TMEM lanes 32(w%4)..+31 (its lane quarter); thread t
-// stores row q's word for slot k at column k*32 + q of lane 32(w%4)+t.  Each
+// stores row q's word for slot k at column q*8 + k of lane 32(w%4)+t, so a
+// flush reads two rows' 8 slots with one 16-column load (16 registers).  Each
 // CTA allocates 256 columns, so two CTAs (two clock-loop warps per SMSP) fit.
 // ---------------------------------------------------------------------------
 constexpr uint32_t TMEM_COLS = 256;
@@ -235,25 +240,29 @@ __device__ __forceinline__ void tmem_dealloc_cta(uint32_t base)
         asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(base), "n"(TMEM_COLS) : "memory");
 }
 
-// 16 consecutive columns of this thread's lane <- x[0..15]
-__device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&x)[16])
+// column taddr + OFF of this thread's lane <- v (one uniform base register,
+// immediate column offsets: STTM tmem[UR + imm])
+template <int OFF>
+__device__ __forceinline__ void tmem_st1(uint32_t taddr, uint32_t v)
 {
-    asm volatile(
-        "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, "
-        "%14, %15, %16};" ::"r"(taddr),
-        "r"(x[0]), "r"(x[1]), "r"(x[2]), "r"(x[3]), "r"(x[4]), "r"(x[5]), "r"(x[6]), "r"(x[7]), "r"(x[8]),
-        "r"(x[9]), "r"(x[10]), "r"(x[11]), "r"(x[12]), "r"(x[13]), "r"(x[14]), "r"(x[15])
-        : "memory");
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0+%2], {%1};" ::"r"(taddr), "r"(v), "n"(OFF) : "memory");
+}
+template <int H, int... Q>
+__device__ __forceinline__ void tmem_st_rows(uint32_t base, const uint32_t (&x)[16], std::integer_sequence<int, Q...>)
+{
+    (tmem_st1<(16 * H + Q) * 8>(base, x[Q]), ...);
 }
 
-// v[0..7] <- 8 consecutive columns of this thread's lane (load + wait in one
+// v[0..15] <- 16 consecutive columns of this thread's lane (load + wait in one
 // asm block, so no use of v can be scheduled before the data has arrived)
-__device__ __forceinline__ void tmem_ld8(uint32_t taddr, uint32_t (&v)[8])
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&v)[16])
 {
     asm volatile(
-        "tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];\n\t"
+        "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, "
+        "%15}, [%16];\n\t"
         "tcgen05.wait::ld.sync.aligned;"
-        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7])
+        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+          "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
         : "r"(taddr)
         : "memory");
 }
@@ -261,7 +270,7 @@ __device__ __forceinline__ void tmem_ld8(uint32_t taddr, uint32_t (&v)[8])
 __device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 
 // Transpose 32 z words held in registers and park the row words of slot k in
-// TMEM columns k*32 + q (tm = this warp's lane-quarter base address).
+// TMEM columns q*8 + k (tm = this warp's lane-quarter base address).
 template <bool MSB_FIRST>
 __device__ __forceinline__ void rowmajor_transpose_tmem(const uint32_t (&z)[32], uint32_t tm, uint32_t k)
 {
@@ -272,7 +281,10 @@ __device__ __forceinline__ void rowmajor_transpose_tmem(const uint32_t (&z)[32],
 #pragma unroll
         for (int q = 0; q < 16; ++q) x[q] = __byte_perm(z[q ^ X], z[(q + 16) ^ X], h == 0 ? 0x5410 : 0x7632);
         bt_transpose16(x);
-        tmem_st16(tm + k * 32 + 16 * h, x);
+        if (h == 0)
+            tmem_st_rows<0>(tm + k, x, std::make_integer_sequence<int, 16>{});
+        else
+            tmem_st_rows<1>(tm + k, x, std::make_integer_sequence<int, 16>{});
     }
 }
 // The same from 32 z words staged in shared memory ([t][lane], zs = lane's column).
@@ -287,7 +299,10 @@ __device__ __forceinline__ void rowmajor_transpose_smem_tmem(const uint32_t* zs,
         for (int q = 0; q < 16; ++q)
             x[q] = __byte_perm(zs[(q ^ X) * 32], zs[((q + 16) ^ X) * 32], h == 0 ? 0x5410 : 0x7632);
         bt_transpose16(x);
-        tmem_st16(tm + k * 32 + 16 * h, x);
+        if (h == 0)
+            tmem_st_rows<0>(tm + k, x, std::make_integer_sequence<int, 16>{});
+        else
+            tmem_st_rows<1>(tm + k, x, std::make_integer_sequence<int, 16>{});
     }
 }
 
@@ -302,40 +317,35 @@ __device__ __forceinline__ void rowmajor_store_tmem(uint32_t tm, uint8_t* row0, 
     const uint64_t align = reinterpret_cast<uintptr_t>(p) | row_bytes;
     const bool full = k_lo == 0 && k_hi == 7;
 #pragma unroll 1
-    for (uint32_t q0 = 0; q0 < 32; q0 += 8) {
-        uint32_t v[8][8];  // [slot][row]
+    for (uint32_t q0 = 0; q0 < 32; q0 += 2) {
+        uint32_t v[16];  // row q0 slots 0..7, row q0+1 slots 0..7
+        tmem_ld16(tm + q0 * 8, v);
 #pragma unroll
-        for (int k = 0; k < 8; ++k) tmem_ld8(tm + k * 32 + q0, v[k]);
-        if (full && (align & 15) == 0) {
+        for (int r = 0; r < 2; ++r) {
+            if (q0 + r >= nvalid) continue;
+            const uint32_t* w = v + 8 * r;
+            uint8_t* d = p + (q0 + r) * row_bytes;
+            if (full && (align & 15) == 0) {
+                __stcs(reinterpret_cast<uint4*>(d), make_uint4(w[0], w[1], w[2], w[3]));
+                __stcs(reinterpret_cast<uint4*>(d) + 1, make_uint4(w[4], w[5], w[6], w[7]));
+            } else if (full && (align & 7) == 0) {
 #pragma unroll
-            for (int r = 0; r < 8; ++r) {
-                if (q0 + r < nvalid) {
-                    uint4* d = reinterpret_cast<uint4*>(p + (q0 + r) * row_bytes);
-                    __stcs(d, make_uint4(v[0][r], v[1][r], v[2][r], v[3][r]));
-                    __stcs(d + 1, make_uint4(v[4][r], v[5][r], v[6][r], v[7][r]));
-                }
-            }
-        } else if (full && (align & 7) == 0) {
+                for (int k = 0; k < 8; k += 2) __stcs(reinterpret_cast<uint2*>(d) + k / 2, make_uint2(w[k], w[k + 1]));
+            } else {
 #pragma unroll
-            for (int r = 0; r < 8; ++r) {
-                if (q0 + r < nvalid) {
-                    uint2* d = reinterpret_cast<uint2*>(p + (q0 + r) * row_bytes);
-#pragma unroll
-                    for (int k = 0; k < 8; k += 2) __stcs(d + k / 2, make_uint2(v[k][r], v[k + 1][r]));
-                }
-            }
-        } else {
-#pragma unroll
-            for (int r = 0; r < 8; ++r) {
-                if (q0 + r < nvalid) {
-                    uint32_t* d = reinterpret_cast<uint32_t*>(p + (q0 + r) * row_bytes);
-#pragma unroll
-                    for (int k = 0; k < 8; ++k)
-                        if (uint32_t(k) >= k_lo && uint32_t(k) <= k_hi) __stcs(d + (k - k_lo), v[k][r]);
-                }
+                for (int k = 0; k < 8; ++k)
+                    if (uint32_t(k) >= k_lo && uint32_t(k) <= k_hi)
+                        __stcs(reinterpret_cast<uint32_t*>(d) + (k - k_lo), w[k]);
             }
         }
     }
+}
+
+__device__ __forceinline__ uint32_t tid_volatile()
+{
+    uint32_t v;
+    asm volatile("mov.u32 %0, %%tid.x;" : "=r"(v));
+    return v;
 }
 
 __device__ __forceinline__ uint32_t laneid_volatile()
@@ -363,6 +373,8 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
     extern __shared__ uint32_t rm_smem[];  // ROW_MAJOR only: NW * rm_warp_words(U, SLOTS, ZREG) (none with TMEM and ZREG)
     __shared__ uint8_t* s_row0[LAYOUT == L_ROW_MAJOR ? BLOCK : 1];
     __shared__ uint32_t s_nvalid[LAYOUT == L_ROW_MAJOR ? BLOCK : 1];
+    __shared__ uint64_t s_b0[LAYOUT == L_ROW_MAJOR ? NW : 1];
+    __shared__ uint32_t s_nblk[LAYOUT == L_ROW_MAJOR ? NW : 1];
     __shared__ uint32_t s_item[NW];
     // Only `s_item` (smem) and the loop counters survive a clock loop; every
     // other per-item value is re-derived afterwards, so the 200 state words
@@ -448,15 +460,22 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
             const uint32_t nvalid = first >= a.n ? 0u : uint32_t(a.n - first < 32 ? a.n - first : 32);
             s_row0[threadIdx.x] = static_cast<uint8_t*>(a.out) + (nvalid ? first : 0) * a.row_bytes;
             s_nvalid[threadIdx.x] = nvalid;
-            uint32_t* zs = rm_smem + (threadIdx.x >> 5) * (TMEM ? ZS_WORDS : rm_warp_words(U, SLOTS, ZREG)) + lane;
-            uint32_t* os = zs + (U == 32 && ZREG ? 0 : ZS_WORDS);
-            const uint64_t b0 = clk_begin >> 5;  // call-relative index of the first 32-clock block
-            const uint32_t nblk = nclk >> 5;
+            // per-warp block context in smem: only `blk` stays in a register
+            // across the clock loop (MICKEY's 200 state words leave ~40)
+            if (lane == 0) {
+                s_b0[threadIdx.x >> 5] = clk_begin >> 5;  // call-relative index of the item's first block
+                s_nblk[threadIdx.x >> 5] = uint32_t(nclk >> 5);
+            }
+            __syncwarp();
             constexpr uint32_t NSLOT = TMEM ? 8 : SLOTS;
+            constexpr int WW = TMEM ? ZS_WORDS : rm_warp_words(U, SLOTS, ZREG);
+            // re-derived after every clock loop from non-CSE-able special registers
+            auto zs_ptr = [&]() { return rm_smem + (tid_volatile() >> 5) * WW + laneid_volatile(); };
+            auto os_ptr = [&]() { return zs_ptr() + (U == 32 && ZREG ? 0 : ZS_WORDS); };
 #pragma unroll 1
-            for (uint32_t blk = 0; blk < nblk; ++blk) {
-                const uint64_t B = b0 + blk;
-                const uint32_t k = uint32_t(B & (NSLOT - 1));
+            for (uint32_t blk = 0;; ++blk) {
+                const uint32_t nblk = *reinterpret_cast<volatile uint32_t*>(&s_nblk[tid_volatile() >> 5]);
+                if (blk >= nblk) break;
                 if constexpr (U == 32 && ZREG) {
                     // one 32-clock block per iteration: keep the z words in
                     // registers and transpose them there (no z staging in smem)
@@ -466,11 +485,14 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
                         zr[u] = c.z();
                         c.clock();
                     }
+                    const uint64_t B = *reinterpret_cast<volatile uint64_t*>(&s_b0[tid_volatile() >> 5]) + blk;
+                    const uint32_t k = uint32_t(B & (NSLOT - 1));
                     if constexpr (TMEM)
                         rowmajor_transpose_tmem<C::MSB_FIRST>(zr, tm_addr(), k);
                     else
-                        rowmajor_transpose_regs<C::MSB_FIRST, SLOTS>(zr, os, k);
+                        rowmajor_transpose_regs<C::MSB_FIRST, SLOTS>(zr, os_ptr(), k);
                 } else {
+                    uint32_t* zs = zs_ptr();
 #pragma unroll 1
                     for (uint32_t kk = 0; kk < 32; kk += U) {
 #pragma unroll
@@ -479,18 +501,23 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
                             c.clock();
                         }
                     }
+                    const uint64_t B = *reinterpret_cast<volatile uint64_t*>(&s_b0[tid_volatile() >> 5]) + blk;
+                    const uint32_t k = uint32_t(B & (NSLOT - 1));
                     if constexpr (TMEM)
-                        rowmajor_transpose_smem_tmem<C::MSB_FIRST>(zs, tm_addr(), k);
+                        rowmajor_transpose_smem_tmem<C::MSB_FIRST>(zs_ptr(), tm_addr(), k);
                     else
-                        rowmajor_transpose<C::MSB_FIRST, SLOTS>(zs, os, k);
+                        rowmajor_transpose<C::MSB_FIRST, SLOTS>(zs_ptr(), os_ptr(), k);
                 }
+                const uint64_t B = *reinterpret_cast<volatile uint64_t*>(&s_b0[tid_volatile() >> 5]) + blk;
+                const uint32_t k = uint32_t(B & (NSLOT - 1));
                 if (k == NSLOT - 1 || blk + 1 == nblk) {
                     const uint32_t k_lo = k - (blk < k ? blk : k);
+                    const uint32_t t = tid_volatile();
                     if constexpr (TMEM)
-                        rowmajor_store_tmem(tm_addr(), s_row0[threadIdx.x], a.row_bytes, s_nvalid[threadIdx.x], k_lo, k,
+                        rowmajor_store_tmem(tm_addr(), s_row0[t], a.row_bytes, s_nvalid[t], k_lo, k,
                                             (B - (k - k_lo)) * 4);
                     else
-                        rowmajor_store<SLOTS>(os, s_row0[threadIdx.x], a.row_bytes, s_nvalid[threadIdx.x], k_lo, k,
+                        rowmajor_store<SLOTS>(os_ptr(), s_row0[t], a.row_bytes, s_nvalid[t], k_lo, k,
                                               (B - (k - k_lo)) * 4);
                 }
             }

@@ -21,6 +21,7 @@ struct Lfsr128 {
     static constexpr int NSTATE = 128;
     static constexpr bool MSB_FIRST = true;
     static constexpr int U_DEFAULT = 32, U_ALT0 = 8, U_ALT1 = 16;
+    static constexpr bool RM_TMEM = false, RM_SEGMENTED = true;
     uint32_t s[128];
 
     __device__ __forceinline__ void load(const uint32_t* st, uint64_t Gp, uint64_t g)

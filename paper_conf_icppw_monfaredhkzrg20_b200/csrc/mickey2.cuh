@@ -116,6 +116,10 @@ struct Mickey2 {
     // clocks per loop iteration: 4 keeps the loop (21 KB of SASS) in the
     // instruction cache; 2 and 8 are built for sweeps ("unroll" option)
     static constexpr int U_DEFAULT = 4, U_ALT0 = 2, U_ALT1 = 8;
+    // ROW_MAJOR default: the plain clock kernel with row segments staged in
+    // TMEM, two CTAs per SM, one work item per warp-unit (0.935 of the ALU
+    // roofline vs 0.904 for the smem warp-specialised kernel)
+    static constexpr bool RM_TMEM = true, RM_SEGMENTED = false;
     uint32_t r[100], s[100];
 
     // State carry (SURVEY step a-5).  The row pointer goes through opaque()

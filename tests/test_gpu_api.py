@@ -51,10 +51,12 @@ def test_zero_bits_is_noop(cipher):
 @pytest.mark.parametrize("cipher,opts", [
     ("mickey2", {"unroll": 2}), ("mickey2", {"unroll": 8}), ("mickey2", {"sched": 0}),
     ("mickey2", {"ctas_per_sm": 2}), ("mickey2", {"rm_ws": 0}), ("mickey2", {"rm_ws": 1, "seg_clocks": 512}),
+    ("mickey2", {"rm_ws": 1}), ("mickey2", {"rm_tmem": 0}), ("mickey2", {"rm_tmem": 1, "seg_clocks": 384}),
     ("grain", {"unroll": 8}), ("grain", {"unroll": 16}), ("grain", {"rm_ws": 1}), ("grain", {"sched": 0}),
     ("grain", {"ctas_per_sm": 1, "seg_clocks": 256}),
-    ("grain", {"rm_slots": 8}), ("grain", {"rm_slots": 4, "rm_zreg": 0}), ("grain", {"rm_slots": 8, "rm_zreg": 0}),
-    ("grain", {"rm_slots": 4, "ctas_per_sm": 2, "seg_clocks": 384}),
+    ("grain", {"rm_tmem": 0}), ("grain", {"rm_tmem": 0, "rm_slots": 4, "rm_zreg": 0}),
+    ("grain", {"rm_tmem": 0, "rm_slots": 8, "rm_zreg": 0}),
+    ("grain", {"rm_tmem": 0, "rm_slots": 4, "ctas_per_sm": 2, "seg_clocks": 384}),
     ("mickey2", {"rm_ws": 0, "rm_slots": 4}), ("mickey2", {"rm_ws": 0, "rm_slots": 4, "seg_clocks": 160}),
     ("aes128ctr", {"ctas_per_sm": 1}), ("aes128ctr", {"rm_ws": 0}), ("aes128ctr", {"seg_clocks": 4096}),
 ])
@@ -80,7 +82,7 @@ def test_option_validation():
     keys, ivs = inputs.make_inputs("grain", 32)
     g = bsrng.Generator("grain", keys, ivs)
     for k, v in (("unroll", 4), ("sched", 2), ("seg_clocks", 33), ("ctas_per_sm", 99), ("rm_ws", 5),
-                 ("rm_slots", 2), ("rm_zreg", 3), ("rm_tmem", 2)):
+                 ("rm_slots", 2), ("rm_zreg", 3), ("rm_tmem", 2), ("init_fused", 2)):
         with pytest.raises(bsrng.BsrngError) as e:
             g.set_option(k, v)
         assert e.value.code == bsrng.EINVAL
@@ -156,3 +158,26 @@ def test_rm_tmem_staging_bit_exact(cipher, opts, bits):
     got2 = g.generate_host(256, "row_major")
     want2 = _want(cipher, keys, ivs, bits + 256)[:, bits // 8:]
     assert np.array_equal(got2, want2)
+
+
+@pytest.mark.parametrize("cipher", ["mickey2", "grain", "aes128ctr", "lfsr128"])
+@pytest.mark.parametrize("init_fused", [1, 0])
+def test_init_paths_keystream(cipher, init_fused):
+    """Both initialisation paths (slicing fused into the init kernel / the
+    ballot slice kernels) give the oracle's keystream after a rekey, at a
+    ragged n spanning several warp-units."""
+    n, bits = 32 * 70 + 17, 512
+    if cipher == "lfsr128":
+        keys, _ = inputs.make_inputs(cipher, n)
+        want = oracle.lfsr128_keystream_batch(keys, bits)
+        g = bsrng.Generator(cipher, inputs.make_inputs(cipher, n, seed=5)[0], None)
+        g.set_option("init_fused", init_fused)
+        g.rekey(keys, None)
+    else:
+        keys, ivs = inputs.make_inputs(cipher, n)
+        want = _want(cipher, keys, ivs, bits)
+        k0, v0 = inputs.make_inputs(cipher, n, seed=5)
+        g = _gen(cipher, k0, v0)
+        g.set_option("init_fused", init_fused)
+        g.rekey(inputs.aes_key() if cipher == "aes128ctr" else keys, ivs)
+    assert np.array_equal(g.generate_host(bits, "row_major"), want)
