@@ -35,13 +35,24 @@ sys.path.insert(0, ROOT)
 N_DEFAULT = 1 << 22
 BITS_DEFAULT = 1 << 20
 # Algorithmic LOP3 per keystream bit position per 32-instance group (DESIGN.md
-# sec. 5): MICKEY 2.0 327 per clock (output op included);
+# sec. 5): MICKEY 2.0 327 per clock in the spec's Galois form (SURVEY App. D,
+# output op included), 304 with the R reduction deferred over K = 4-clock
+# blocks (315.5 at K = 2; mickey2.cuh clock_lazy, DESIGN.md sec. 5 item 10);
 # Grain v1 37 per clock (f 3 + g 25 + h/z 9) + 1 to fold into the checksum;
 # AES-128-CTR 17280 per 32-block encryption (4096 bit positions) + 64 for the
 # checksum XOR tree.
-def lop3_per_bit(cipher, mode):
+MICKEY2_GALOIS_OPS = 327.0
+MICKEY2_OPS_BY_BLOCK = {1: 327.0, 2: 315.5, 4: 304.0}
+
+
+def mickey2_block(unroll):
+    """Deferred-reduction block K for a U-clock loop body (Mickey2::block_k)."""
+    return 4 if unroll % 4 == 0 else 2 if unroll % 2 == 0 else 1
+
+
+def lop3_per_bit(cipher, mode, unroll=None):
     if cipher == "mickey2":
-        return 327.0
+        return MICKEY2_OPS_BY_BLOCK[mickey2_block(unroll or 4)]
     if cipher == "grain":
         return 38.0 if mode == "consume" else 37.0
     if cipher == "lfsr128":
@@ -393,13 +404,19 @@ def run_ours(args, rank, world, local_rank):
                 "note": "rekey = slice kernels + preclock kernel (+ H2D for e2e)"}
 
     def roofline(kern_ms_per_step, clocks, mode):
-        lop3 = lop3_per_bit(args.cipher, mode) * (n // 32) * bits  # algorithmic LOP3 per step, dominant kernel
+        unroll = dict(kv.split("=", 1) for kv in args.opt).get("unroll")
+        ops = lop3_per_bit(args.cipher, mode, int(unroll) if unroll else None)
+        lop3 = ops * (n // 32) * bits  # algorithmic LOP3 per step, dominant kernel
         achieved = lop3 / (kern_ms_per_step * 1e-3) / 1e12
         peak = nsm * ALU_LANES_PER_SM_CLK * sm_max * 1e6 / 1e12
         out = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TLOP3/s", "frac": achieved / peak,
                "peak_basis": f"{nsm} SMs x {ALU_LANES_PER_SM_CLK} LOP3 lanes/clk x sm_max {sm_max:.0f} MHz "
                              "(B300_MICROARCH alu pipe rt=2/SMSP; DESIGN.md)",
                "traffic": None}
+        if args.cipher == "mickey2":
+            out["ops_per_clock"] = ops
+            out["galois_ops_per_clock"] = MICKEY2_GALOIS_OPS
+            out["frac_vs_galois_count"] = out["frac"] * MICKEY2_GALOIS_OPS / ops
         if clocks and clocks.get("sm_mhz"):
             out["frac_at_sampled_clock"] = achieved / (nsm * ALU_LANES_PER_SM_CLK * clocks["sm_mhz"] * 1e6 / 1e12)
         return out

@@ -27,11 +27,64 @@
 //              32-bit word per instance row.
 #pragma once
 #include <cstdint>
+#include <type_traits>
 #include <utility>
 
 #include "bitslice.cuh"
 
 namespace bsk {
+
+// Per-clock calls of a U-clock loop body.  A cipher with a multi-clock
+// schedule (MICKEY 2.0's deferred R reduction, mickey2.cuh) declares
+// block_k(U) and clocks J = 0..K-1 of each K-clock block are compile-time
+// phases (z_at / z_acc_at / clock_at); any other cipher uses z / z_acc / clock.
+template <class C, class = void>
+struct ks_phased : std::false_type {};
+template <class C>
+struct ks_phased<C, std::void_t<decltype(C::block_k(1))>> : std::true_type {};
+template <class C, int U>
+__host__ __device__ constexpr int ks_block()
+{
+    if constexpr (ks_phased<C>::value)
+        return C::block_k(U);
+    else
+        return 1;
+}
+template <int J, int K, class C>
+__device__ __forceinline__ uint32_t ks_z(const C& c)
+{
+    if constexpr (K > 1)
+        return c.template z_at<J, K>();
+    else
+        return c.z();
+}
+template <int J, int K, class C>
+__device__ __forceinline__ uint32_t ks_z_acc(const C& c, uint32_t acc)
+{
+    if constexpr (K > 1)
+        return c.template z_acc_at<J, K>(acc);
+    else
+        return c.z_acc(acc);
+}
+template <int J, int K, class C>
+__device__ __forceinline__ void ks_clock(C& c)
+{
+    if constexpr (K > 1)
+        c.template clock_at<J, K>();
+    else
+        c.clock();
+}
+template <class F, int... I>
+__device__ __forceinline__ void static_for_impl(F&& f, std::integer_sequence<int, I...>)
+{
+    (f(std::integral_constant<int, I>{}), ...);
+}
+// f(integral_constant<int, i>) for i = 0..N-1, fully unrolled
+template <int N, class F>
+__device__ __forceinline__ void static_for(F&& f)
+{
+    static_for_impl(f, std::make_integer_sequence<int, N>{});
+}
 
 enum : int { L_ROW_MAJOR = 0, L_SLICED = 1, L_CHECKSUM = 2 };
 
@@ -369,6 +422,8 @@ template <class C, int LAYOUT, int U, int BLOCK, int SLOTS = 8, bool ZREG = true
 __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
 {
     static_assert(32 % U == 0, "U must divide 32");
+    constexpr int KB = ks_block<C, U>();  // clocks per cipher schedule block
+    static_assert(U % KB == 0, "the loop body must hold whole schedule blocks");
     constexpr int NW = BLOCK / 32;
     extern __shared__ uint32_t rm_smem[];  // ROW_MAJOR only: NW * rm_warp_words(U, SLOTS, ZREG) (none with TMEM and ZREG)
     __shared__ uint8_t* s_row0[LAYOUT == L_ROW_MAJOR ? BLOCK : 1];
@@ -434,11 +489,11 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
         if (LAYOUT == L_CHECKSUM) {
 #pragma unroll 1
             for (uint32_t it = nclk / U; it != 0; --it) {
-#pragma unroll
-                for (int u = 0; u < U; ++u) {
-                    acc = c.z_acc(acc);
-                    c.clock();
-                }
+                static_for<U>([&](auto u) {
+                    constexpr int J = decltype(u)::value % KB;
+                    acc = ks_z_acc<J, KB>(c, acc);
+                    ks_clock<J, KB>(c);
+                });
             }
         } else if (LAYOUT == L_SLICED) {
             const uint32_t m = lane_mask(a, g);
@@ -448,12 +503,12 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
             const uint64_t stride = g < a.G ? a.G : 0;
 #pragma unroll 1
             for (uint32_t it = nclk / U; it != 0; --it) {
-#pragma unroll
-                for (int u = 0; u < U; ++u) {
-                    __stcs(o, c.z() & m);
+                static_for<U>([&](auto u) {
+                    constexpr int J = decltype(u)::value % KB;
+                    __stcs(o, ks_z<J, KB>(c) & m);
                     o += stride;
-                    c.clock();
-                }
+                    ks_clock<J, KB>(c);
+                });
             }
         } else {  // ROW_MAJOR
             const uint64_t first = g * 32u;
@@ -480,11 +535,11 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
                     // one 32-clock block per iteration: keep the z words in
                     // registers and transpose them there (no z staging in smem)
                     uint32_t zr[32];
-#pragma unroll
-                    for (int u = 0; u < 32; ++u) {
-                        zr[u] = c.z();
-                        c.clock();
-                    }
+                    static_for<32>([&](auto u) {
+                        constexpr int J = decltype(u)::value % KB;
+                        zr[decltype(u)::value] = ks_z<J, KB>(c);
+                        ks_clock<J, KB>(c);
+                    });
                     const uint64_t B = *reinterpret_cast<volatile uint64_t*>(&s_b0[tid_volatile() >> 5]) + blk;
                     const uint32_t k = uint32_t(B & (NSLOT - 1));
                     if constexpr (TMEM)
@@ -495,11 +550,11 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
                     uint32_t* zs = zs_ptr();
 #pragma unroll 1
                     for (uint32_t kk = 0; kk < 32; kk += U) {
-#pragma unroll
-                        for (int u = 0; u < U; ++u) {
-                            zs[(kk + u) * 32] = c.z();
-                            c.clock();
-                        }
+                        static_for<U>([&](auto u) {
+                            constexpr int J = decltype(u)::value % KB;
+                            zs[(kk + decltype(u)::value) * 32] = ks_z<J, KB>(c);
+                            ks_clock<J, KB>(c);
+                        });
                     }
                     const uint64_t B = *reinterpret_cast<volatile uint64_t*>(&s_b0[tid_volatile() >> 5]) + blk;
                     const uint32_t k = uint32_t(B & (NSLOT - 1));

@@ -81,8 +81,8 @@ __device__ __forceinline__ void s_update(uint32_t (&ns)[100], const uint32_t (&s
 // R is updated in place top-down (old r_i is read only by r'_i and r'_{i+1});
 // S goes through a renamed array (every old s_i is read by three updates), which
 // after full unrolling is pure register renaming.
-template <bool MIX>
-__device__ __forceinline__ void clock_kg(uint32_t (&r)[100], uint32_t (&s)[100], uint32_t in)
+template <bool MIX, int NR>
+__device__ __forceinline__ void clock_kg(uint32_t (&r)[NR], uint32_t (&s)[100], uint32_t in)
 {
     const uint32_t ctl_r = s[34] ^ r[67];
     const uint32_t ctl_s = s[67] ^ r[33];
@@ -104,6 +104,190 @@ __device__ __forceinline__ void clock_kg(uint32_t (&r)[100], uint32_t (&s)[100],
     for (int i = 0; i < 100; ++i) s[i] = ns[i];
 }
 
+// ---------------------------------------------------------------------------
+// Keystream clocks with the Galois reduction of R deferred over a block of K
+// clocks (K = 2, 4 or 8; B200 design, not the paper's).
+//
+// In polynomial form (spec [5]: r'_i = r_{i-1} ^ [i in RTAPS] r99 ^ (ctlR & r_i))
+// the R clock is R' = (x + ctlR) * R mod p(x), p(x) = x^100 + sum_{t in RTAPS}
+// x^t, lane by lane.  Multiplication commutes with the reduction, so within a
+// block we keep an unreduced P == R (mod p) whose degree grows by one per
+// clock: P' = (x + ctlR) * P costs one LOP3 per position and no feedback taps
+// (the new top word is a rename).  At the block's end the K overflow words
+// h_m = P_{100+m} are folded back, h_m * x^(100+m) mod p = h_m * Q_m(x): each
+// low position q receives the XOR of the h_m with q in Q_m.  Pairs of h words
+// are pre-combined (h_0^h_1, h_2^h_3, ...), so a position takes at most one
+// operand per pair: one LOP3 per position at K = 4 instead of one per tap per
+// clock.  The three taps the clock reads mid-block (r0 for z, r33 for
+// CONTROL_BIT_S, r67 for CONTROL_BIT_R) add their pending h_m terms explicitly.
+//
+// Ops per clock for R at K = 4: 101.5 (shift) + 1.25 (tap corrections) + 23.25
+// (reduction incl. 2 pair combos) = 126 vs 149 in Galois form, so a keystream
+// clock is 304 LOP3 instead of 327 (`lazy_ops_per_clock`).
+// Bit-exactness: at every block boundary P is fully reduced and equals the
+// spec's R (the state carry and the parity tests see only reduced states).
+// ---------------------------------------------------------------------------
+constexpr int KMAX = 8;  // largest block; Q_0..Q_7
+
+struct QTab {
+    uint32_t w[KMAX][4];
+};
+// Q_m = x^(100+m) mod p(x) as bit masks (bit q of word q/32)
+__host__ __device__ constexpr QTab make_qtab()
+{
+    QTab t{};
+    uint32_t cur[4] = {0x1279327Bu, 0xB5546660u, 0xDF87818Fu, 0x00000003u};  // x^100 = sum RTAPS x^t
+    for (int m = 0; m < KMAX; ++m) {
+        for (int i = 0; i < 4; ++i) t.w[m][i] = cur[i];
+        const uint32_t carry = (cur[3] >> 3) & 1u;  // bit 99
+        cur[3] = ((cur[3] << 1) | (cur[2] >> 31)) & 0xFu;
+        cur[2] = (cur[2] << 1) | (cur[1] >> 31);
+        cur[1] = (cur[1] << 1) | (cur[0] >> 31);
+        cur[0] = cur[0] << 1;
+        if (carry) {
+            cur[0] ^= 0x1279327Bu;
+            cur[1] ^= 0xB5546660u;
+            cur[2] ^= 0xDF87818Fu;
+            cur[3] ^= 0x00000003u;
+        }
+    }
+    return t;
+}
+__host__ __device__ constexpr bool qbit(int m, int q)
+{
+    return (make_qtab().w[m][q >> 5] >> (q & 31)) & 1u;
+}
+// pending words m < J that feed position q, and the i-th of them
+__host__ __device__ constexpr int n_terms(int q, int J)
+{
+    int n = 0;
+    for (int m = 0; m < J; ++m) n += qbit(m, q) ? 1 : 0;
+    return n;
+}
+__host__ __device__ constexpr int term_m(int q, int J, int i)
+{
+    for (int m = 0; m < J; ++m)
+        if (qbit(m, q) && i-- == 0) return m;
+    return -1;
+}
+
+constexpr int RN = 100 + KMAX;  // R register words incl. pending positions
+constexpr uint32_t XOR2 = 0x3Cu, XOR3 = 0x96u, AND2 = 0xC0u;
+
+// XOR of: e[0..NE-1], r[Q] and the pending terms of position Q at phase J
+// (the true spec bit r_Q mid-block), two operands per LOP3.
+template <int Q, int J, int NE, int K>
+__device__ __forceinline__ uint32_t opnd(const uint32_t (&e)[NE], const uint32_t (&r)[RN])
+{
+    if constexpr (K < NE)
+        return e[K];
+    else if constexpr (K == NE)
+        return r[Q];
+    else
+        return r[100 + term_m(Q, J, K - NE - 1)];
+}
+template <int Q, int J, int NE, int K, int NT>
+__device__ __forceinline__ uint32_t fold(uint32_t v, const uint32_t (&e)[NE], const uint32_t (&r)[RN])
+{
+    if constexpr (K + 1 < NT)
+        return fold<Q, J, NE, K + 2, NT>(lop3<XOR3>(v, opnd<Q, J, NE, K>(e, r), opnd<Q, J, NE, K + 1>(e, r)), e, r);
+    else if constexpr (K < NT)
+        return lop3<XOR2>(v, opnd<Q, J, NE, K>(e, r), 0u);
+    else
+        return v;
+}
+template <int Q, int J, int NE>
+__device__ __forceinline__ uint32_t xor_true(const uint32_t (&e)[NE], const uint32_t (&r)[RN])
+{
+    constexpr int NT = NE + 1 + n_terms(Q, J);
+    return fold<Q, J, NE, 1, NT>(opnd<Q, J, NE, 0>(e, r), e, r);
+}
+
+// End-of-block reduction: r[q] ^= sum_{m < K, q in Q_m} h_m, h_m = r[100+m].
+// Operand of pair p for position q: h_{2p}, h_{2p+1} or their pre-combined XOR.
+template <int K>
+__device__ __forceinline__ uint32_t pair_opnd(const uint32_t (&r)[RN], const uint32_t (&cmb)[KMAX / 2], int p, int q)
+{
+    const bool a = qbit(2 * p, q), b = K > 2 * p + 1 && qbit(2 * p + 1, q);
+    return a && b ? cmb[p] : a ? r[100 + 2 * p] : r[101 + 2 * p];
+}
+__host__ __device__ constexpr bool pair_used(int K, int p, int q)
+{
+    return qbit(2 * p, q) || (K > 2 * p + 1 && qbit(2 * p + 1, q));
+}
+__host__ __device__ constexpr int n_pairs_used(int K, int q)
+{
+    int n = 0;
+    for (int p = 0; p < (K + 1) / 2; ++p) n += pair_used(K, p, q) ? 1 : 0;
+    return n;
+}
+__host__ __device__ constexpr int pair_i(int K, int q, int i)
+{
+    for (int p = 0; p < (K + 1) / 2; ++p)
+        if (pair_used(K, p, q) && i-- == 0) return p;
+    return -1;
+}
+__host__ __device__ constexpr bool combo_needed(int K, int p)
+{
+    if (K <= 2 * p + 1) return false;
+    for (int q = 0; q < 100; ++q)
+        if (qbit(2 * p, q) && qbit(2 * p + 1, q)) return true;
+    return false;
+}
+template <int K, int Q, int I, int N>
+__device__ __forceinline__ uint32_t red_fold(uint32_t v, const uint32_t (&r)[RN], const uint32_t (&cmb)[KMAX / 2])
+{
+    if constexpr (I + 1 < N)
+        return red_fold<K, Q, I + 2, N>(
+            lop3<XOR3>(v, pair_opnd<K>(r, cmb, pair_i(K, Q, I), Q), pair_opnd<K>(r, cmb, pair_i(K, Q, I + 1), Q)), r,
+            cmb);
+    else if constexpr (I < N)
+        return lop3<XOR2>(v, pair_opnd<K>(r, cmb, pair_i(K, Q, I), Q), 0u);
+    else
+        return v;
+}
+template <int K, int... Q>
+__device__ __forceinline__ void reduce(uint32_t (&r)[RN], std::integer_sequence<int, Q...>)
+{
+    uint32_t cmb[KMAX / 2];
+#pragma unroll
+    for (int p = 0; p < KMAX / 2; ++p) cmb[p] = 0u;
+    if constexpr (combo_needed(K, 0)) cmb[0] = lop3<XOR2>(r[100], r[101], 0u);
+    if constexpr (combo_needed(K, 1)) cmb[1] = lop3<XOR2>(r[102], r[103], 0u);
+    if constexpr (combo_needed(K, 2)) cmb[2] = lop3<XOR2>(r[104], r[105], 0u);
+    if constexpr (combo_needed(K, 3)) cmb[3] = lop3<XOR2>(r[106], r[107], 0u);
+    ((r[Q] = red_fold<K, Q, 0, n_pairs_used(K, Q)>(r[Q], r, cmb)), ...);
+}
+
+// The S half of CLOCK_KG (keystream mode), given CONTROL_BIT_S.
+__device__ __forceinline__ void s_clock(uint32_t (&s)[100], uint32_t ctl_s)
+{
+    const uint32_t fb_s = s[99];
+    const uint32_t fb_s0 = fb_s & ~ctl_s;
+    const uint32_t fb_s1 = fb_s & ctl_s;
+    uint32_t ns[100];
+    s_update(ns, s, fb_s, fb_s0, fb_s1, std::make_integer_sequence<int, 100>{});
+#pragma unroll
+    for (int i = 0; i < 100; ++i) s[i] = ns[i];
+}
+
+// Keystream clock J (0..K-1) of a K-clock block.  Before it, r[100..99+J]
+// hold the pending overflow words; after clock K-1, R is reduced again.
+template <int J, int K>
+__device__ __forceinline__ void clock_lazy(uint32_t (&r)[RN], uint32_t (&s)[100])
+{
+    static_assert(K >= 2 && K <= KMAX && J < K, "block of 2..8 clocks");
+    const uint32_t e34[1] = {s[34]}, e67[1] = {s[67]};
+    const uint32_t ctl_r = xor_true<67, J, 1>(e34, r);  // s34 ^ r67
+    const uint32_t ctl_s = xor_true<33, J, 1>(e67, r);  // s67 ^ r33
+    r[100 + J] = r[99 + J];                               // top word: rename
+#pragma unroll
+    for (int i = 99 + J; i >= 1; --i) r[i] = lop3<LUT_A_XOR_BC>(r[i - 1], ctl_r, r[i]);
+    r[0] = lop3<AND2>(ctl_r, r[0], 0u);
+    s_clock(s, ctl_s);
+    if constexpr (J == K - 1) reduce<K>(r, std::make_integer_sequence<int, 100>{});
+}
+
 }  // namespace m2
 }  // namespace bsk
 
@@ -120,7 +304,11 @@ struct Mickey2 {
     // TMEM, two CTAs per SM, one work item per warp-unit (0.935 of the ALU
     // roofline vs 0.904 for the smem warp-specialised kernel)
     static constexpr bool RM_TMEM = true, RM_SEGMENTED = false;
-    uint32_t r[100], s[100];
+    // r[100..107]: pending overflow words of the deferred R reduction
+    // (clock_at); only positions 0..99 are state between blocks
+    uint32_t r[m2::RN], s[100];
+    // clocks per deferred-reduction block for a U-clock loop body
+    static constexpr int block_k(int U) { return U % 4 == 0 ? 4 : U % 2 == 0 ? 2 : 1; }
 
     // State carry (SURVEY step a-5).  The row pointer goes through opaque()
     // so the 200 load addresses are not kept live across the clock loop for
@@ -145,6 +333,24 @@ struct Mickey2 {
     __device__ __forceinline__ uint32_t z() const { return r[0] ^ s[0]; }
     __device__ __forceinline__ uint32_t z_acc(uint32_t acc) const { return acc ^ r[0] ^ s[0]; }
     __device__ __forceinline__ void clock() { m2::clock_kg<false>(r, s, 0u); }
+    // clock J of a K-clock deferred-reduction block (K = block_k(U) > 1)
+    template <int J, int K>
+    __device__ __forceinline__ uint32_t z_at() const
+    {
+        const uint32_t e[1] = {s[0]};
+        return m2::xor_true<0, J, 1>(e, r);
+    }
+    template <int J, int K>
+    __device__ __forceinline__ uint32_t z_acc_at(uint32_t acc) const
+    {
+        const uint32_t e[2] = {acc, s[0]};
+        return m2::xor_true<0, J, 2>(e, r);
+    }
+    template <int J, int K>
+    __device__ __forceinline__ void clock_at()
+    {
+        m2::clock_lazy<J, K>(r, s);
+    }
 };
 
 // Initialisation (SURVEY step a-2, spec [5]): R = S = 0,

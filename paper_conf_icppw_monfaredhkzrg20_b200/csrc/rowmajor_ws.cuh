@@ -68,6 +68,8 @@ template <class C, int U>
 __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const KsArgs a)
 {
     static_assert(32 % U == 0, "U must divide 32");
+    constexpr int KB = ks_block<C, U>();
+    static_assert(U % KB == 0, "the loop body must hold whole schedule blocks");
     extern __shared__ uint32_t pair_smem[];  // [NCOMP][2 z blocks + sector buffer]
     __shared__ uint64_t bar_full[ws::NCOMP][2], bar_empty[ws::NCOMP][2];
     __shared__ ws::Meta meta[ws::NCOMP][2];
@@ -124,11 +126,11 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const KsA
                 uint32_t* zb = zbase + b * ws::ZBUF + laneid_volatile();
 #pragma unroll 1
                 for (uint32_t k = 0; k < 32; k += U) {
-#pragma unroll
-                    for (int u = 0; u < U; ++u) {
-                        zb[(k + u) * 32] = c.z();
-                        c.clock();
-                    }
+                    static_for<U>([&](auto u) {
+                        constexpr int J = decltype(u)::value % KB;
+                        zb[(k + decltype(u)::value) * 32] = ks_z<J, KB>(c);
+                        ks_clock<J, KB>(c);
+                    });
                 }
                 if (laneid_volatile() == 0) {
                     const uint64_t B = s_b0[pair] + blk;

@@ -43,6 +43,87 @@ def test_workloads_match_baseline_configs():
 
 
 def test_op_counts():
-    assert bench.lop3_per_bit("mickey2", "consume") == 327
+    assert bench.lop3_per_bit("mickey2", "consume") == 304          # deferred R reduction, K = 4
+    assert bench.lop3_per_bit("mickey2", "consume", unroll=2) == 315.5
+    assert bench.MICKEY2_GALOIS_OPS == 327
     assert bench.lop3_per_bit("grain", "materialise") == 37
     assert abs(bench.lop3_per_bit("aes128ctr", "materialise") * 4096 / 32 - 17280) < 1e-9
+
+
+# --- the deferred Galois reduction of MICKEY 2.0's R (mickey2.cuh clock_lazy) ---
+# RTAPS of the MICKEY 2.0 specification (ref [5]), as tap positions.
+_RTAPS = [0, 1, 3, 4, 5, 6, 9, 12, 13, 16, 19, 20, 21, 22, 25, 28, 37, 38, 41, 42, 45, 46, 50, 52, 54, 56, 58, 60,
+          61, 63, 64, 65, 66, 67, 71, 72, 79, 80, 81, 82, 87, 88, 89, 90, 91, 92, 94, 95, 96, 97]
+
+
+def _q_masks(k):
+    """Q_m = x^(100+m) mod p(x) as 100-bit integers, m < k."""
+    p_low = sum(1 << t for t in _RTAPS)
+    out, cur = [], p_low
+    for _ in range(k):
+        out.append(cur)
+        cur <<= 1
+        if cur >> 100:
+            cur = (cur & ((1 << 100) - 1)) ^ p_low
+    return out
+
+
+def _lazy_ops(k):
+    """LOP3 per clock of the implemented schedule (pairs of overflow words)."""
+    import math
+    if k == 1:
+        return 327.0
+    Q = _q_masks(k)
+    bit = lambda m, q: (Q[m] >> q) & 1
+    shift = sum(100 + j for j in range(k))
+    corr = 0
+    for j in range(k):
+        for q, base in ((67, 2), (33, 2), (0, 3)):
+            t = sum(bit(m, q) for m in range(j))
+            corr += math.ceil((base + t - 1) / 2) - math.ceil((base - 1) / 2)
+    pairs = [[2 * p, 2 * p + 1] if 2 * p + 1 < k else [2 * p] for p in range((k + 1) // 2)]
+    pre = sum(1 for g in pairs if len(g) == 2 and any(bit(g[0], q) and bit(g[1], q) for q in range(100)))
+    red = sum(math.ceil(sum(1 for g in pairs if any(bit(m, q) for m in g)) / 2) for q in range(100))
+    return 327 - 149 + (shift + corr + red + pre) / k
+
+
+def test_mickey2_deferred_reduction_op_counts():
+    for k in (1, 2, 4):
+        assert _lazy_ops(k) == bench.MICKEY2_OPS_BY_BLOCK[k], k
+
+
+def test_mickey2_deferred_reduction_equals_galois_clocking():
+    """(x + c) * R mod p clocked K times unreduced, then folded with Q_m, equals
+    K Galois clocks of the spec (r'_i = r_{i-1} ^ [i in RTAPS] r99 ^ c r_i), with
+    the taps r0 / r33 / r67 read mid-block through their pending terms."""
+    import random
+    rng = random.Random(2020)
+    taps = set(_RTAPS)
+    for k in (2, 4):
+        Q = _q_masks(k)
+        for _ in range(200):
+            R = rng.getrandbits(100)
+            ctl = [rng.getrandbits(1) for _ in range(k)]
+            # Galois (spec) clocks, recording r0/r33/r67 before each clock
+            g, seen_g = R, []
+            for c in ctl:
+                seen_g.append(((g >> 0) & 1, (g >> 33) & 1, (g >> 67) & 1))
+                r99 = (g >> 99) & 1
+                nxt = 0
+                for i in range(100):
+                    v = ((g >> (i - 1)) & 1 if i else 0) ^ (r99 if i in taps else 0) ^ (c & (g >> i) & 1)
+                    nxt |= v << i
+                g = nxt
+            # deferred: P' = (x + c) P, unreduced; taps read with pending terms
+            P, seen_l = R, []
+            for j, c in enumerate(ctl):
+                pend = [(P >> (100 + m)) & 1 for m in range(j)]
+                true = lambda q: ((P >> q) & 1) ^ (sum(pend[m] & ((Q[m] >> q) & 1) for m in range(j)) & 1)
+                seen_l.append((true(0), true(33), true(67)))
+                P = (P << 1) ^ (P if c else 0)
+            low = P & ((1 << 100) - 1)
+            for m in range(k):
+                if (P >> (100 + m)) & 1:
+                    low ^= Q[m]
+            assert P >> (100 + k) == 0
+            assert low == g and seen_l == seen_g

@@ -53,7 +53,7 @@ def main():
                 ms = e0.elapsed_time(e1)
                 best = ms if best is None else min(best, ms)
             tbps = a.n * a.bits / (best * 1e-3) / 1e12
-            lop3 = 327 * (a.n // 32) * a.bits / (best * 1e-3)
+            lop3 = 304 * (a.n // 32) * a.bits / (best * 1e-3)
             frac = lop3 / (nsm * 64 * 1965e6)
             print(json.dumps({"layout": layout, "opts": kv, "ms": round(best, 3), "tbps": round(tbps, 4),
                               "alu_frac_at_1965": round(frac, 4)}), flush=True)

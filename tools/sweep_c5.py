@@ -32,7 +32,8 @@ import torch  # noqa: E402
 
 from paper_conf_icppw_monfaredhkzrg20_b200 import bsrng  # noqa: E402
 
-OPS = {"mickey2": 327.0, "grain": 37.0, "aes128ctr": 17280.0 / 128.0}
+OPS = {"mickey2": 304.0,  # deferred R reduction (327 in Galois form)
+       "grain": 37.0, "aes128ctr": 17280.0 / 128.0}
 PAPER_CLOCKS = (4416, 12992)  # multiples of 32 nearest the paper's 4,400 / 13,000
 
 
