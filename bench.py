@@ -393,9 +393,11 @@ def run_ours(args, rank, world, local_rank):
 
     def init_roofline(rk_ms):
         """a-1 + a-2 (bsrng_rekey) against the same ALU peak: initialisation
-        clocks x ops per clock (MICKEY 260 x 328, Grain 160 x 39; AES-CTR has
-        no initialisation clocks, only slicing + a one-thread key expansion)."""
-        ops = {"mickey2": 260 * 328.0, "grain": 160 * 39.0}.get(args.cipher)
+        clocks x ops per clock (MICKEY 260 x 306 with the deferred R reduction
+        -- 328 in Galois form: 304 - 1 output + u = INPUT_BIT ^ s50 + its XOR
+        into the pending word + FEEDBACK_S --, Grain 160 x 39; AES-CTR has no
+        initialisation clocks, only slicing + a one-thread key expansion)."""
+        ops = {"mickey2": 260 * 306.0, "grain": 160 * 39.0}.get(args.cipher)
         if not ops or rk_ms <= 0:
             return None
         achieved = ops * (n // 32) / (rk_ms * 1e-3) / 1e12

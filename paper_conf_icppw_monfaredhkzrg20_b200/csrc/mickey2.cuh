@@ -259,10 +259,9 @@ __device__ __forceinline__ void reduce(uint32_t (&r)[RN], std::integer_sequence<
     ((r[Q] = red_fold<K, Q, 0, n_pairs_used(K, Q)>(r[Q], r, cmb)), ...);
 }
 
-// The S half of CLOCK_KG (keystream mode), given CONTROL_BIT_S.
-__device__ __forceinline__ void s_clock(uint32_t (&s)[100], uint32_t ctl_s)
+// The S half of CLOCK_KG, given CONTROL_BIT_S and FEEDBACK_S.
+__device__ __forceinline__ void s_clock(uint32_t (&s)[100], uint32_t ctl_s, uint32_t fb_s)
 {
-    const uint32_t fb_s = s[99];
     const uint32_t fb_s0 = fb_s & ~ctl_s;
     const uint32_t fb_s1 = fb_s & ctl_s;
     uint32_t ns[100];
@@ -271,21 +270,43 @@ __device__ __forceinline__ void s_clock(uint32_t (&s)[100], uint32_t ctl_s)
     for (int i = 0; i < 100; ++i) s[i] = ns[i];
 }
 
-// Keystream clock J (0..K-1) of a K-clock block.  Before it, r[100..99+J]
-// hold the pending overflow words; after clock K-1, R is reduced again.
-template <int J, int K>
-__device__ __forceinline__ void clock_lazy(uint32_t (&r)[RN], uint32_t (&s)[100])
+// Clock J (0..K-1) of a K-clock block.  Before it, r[100..99+J] hold the
+// pending overflow words; after clock K-1, R is reduced again.  MIX = the
+// spec's MIXING (initialisation): FEEDBACK_R gains u = INPUT_BIT ^ s50, i.e.
+// R' = (x + c) R + u * sum_{t in RTAPS} x^t = (x + c) R + u * x^100 (mod p), so
+// u is XORed into the pending word at position 100 (one op, not one per tap);
+// FEEDBACK_S = s99 ^ INPUT_BIT.
+template <int J, int K, bool MIX = false>
+__device__ __forceinline__ void clock_lazy(uint32_t (&r)[RN], uint32_t (&s)[100], uint32_t in = 0u)
 {
     static_assert(K >= 2 && K <= KMAX && J < K, "block of 2..8 clocks");
     const uint32_t e34[1] = {s[34]}, e67[1] = {s[67]};
     const uint32_t ctl_r = xor_true<67, J, 1>(e34, r);  // s34 ^ r67
     const uint32_t ctl_s = xor_true<33, J, 1>(e67, r);  // s67 ^ r33
-    r[100 + J] = r[99 + J];                               // top word: rename
+    const uint32_t u = MIX ? lop3<XOR2>(in, s[50], 0u) : 0u;
+    const uint32_t fb_s = MIX ? lop3<XOR2>(s[99], in, 0u) : s[99];
+    if constexpr (MIX && J == 0)
+        r[100] = lop3<XOR2>(r[99], u, 0u);  // top word: rename, + u x^100
+    else
+        r[100 + J] = r[99 + J];             // top word: rename
 #pragma unroll
-    for (int i = 99 + J; i >= 1; --i) r[i] = lop3<LUT_A_XOR_BC>(r[i - 1], ctl_r, r[i]);
+    for (int i = 99 + J; i >= 1; --i) {
+        if (MIX && J > 0 && i == 100)
+            r[i] = lop3<XOR2>(lop3<LUT_A_XOR_BC>(r[i - 1], ctl_r, r[i]), u, 0u);
+        else
+            r[i] = lop3<LUT_A_XOR_BC>(r[i - 1], ctl_r, r[i]);
+    }
     r[0] = lop3<AND2>(ctl_r, r[0], 0u);
-    s_clock(s, ctl_s);
+    s_clock(s, ctl_s, fb_s);
     if constexpr (J == K - 1) reduce<K>(r, std::make_integer_sequence<int, 100>{});
+}
+// four initialisation clocks (MIXING = 1) with input words in[0..3]
+__device__ __forceinline__ void clock4_mix(uint32_t (&r)[RN], uint32_t (&s)[100], const uint32_t (&in)[4])
+{
+    clock_lazy<0, 4, true>(r, s, in[0]);
+    clock_lazy<1, 4, true>(r, s, in[1]);
+    clock_lazy<2, 4, true>(r, s, in[2]);
+    clock_lazy<3, 4, true>(r, s, in[3]);
 }
 
 }  // namespace m2
@@ -437,22 +458,26 @@ __global__ void __launch_bounds__(M2I_BLOCK, 2) m2_init_kernel(const uint8_t* __
     slice_group32<10, 80, true>(raw_iv + g * 320u, [&](int bit, uint32_t w) { sl[bit * M2I_BLOCK] = w; });
     slice_group32<10, 80, true>(raw_k + g * 320u, [&](int bit, uint32_t w) { sl[(80 + bit) * M2I_BLOCK] = w; });
 
-    uint32_t r[100], s[100];
+    // R with the deferred reduction (m2::clock_lazy, 4-clock blocks; reduced
+    // again at every block boundary, so the stored state is the spec's)
+    uint32_t r[m2::RN], s[100];
 #pragma unroll
     for (int i = 0; i < 100; ++i) r[i] = s[i] = 0u;
     const int nin = iv_bits + 80;  // IV clocks, then key clocks: rows 0..iv_bits-1, 80..159
 #pragma unroll 1
     for (int c = 0; c < nin; c += 4) {
+        uint32_t in[4];
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
             const int row = c + u < iv_bits ? c + u : c + u - iv_bits + 80;
-            m2::clock_kg<true>(r, s, sl[row * M2I_BLOCK]);
+            in[u] = sl[row * M2I_BLOCK];
         }
+        m2::clock4_mix(r, s, in);
     }
 #pragma unroll 1
     for (int i = 0; i < 100; i += 4) {
-#pragma unroll
-        for (int u = 0; u < 4; ++u) m2::clock_kg<true>(r, s, 0u);
+        const uint32_t in[4] = {0u, 0u, 0u, 0u};
+        m2::clock4_mix(r, s, in);
     }
     uint32_t* p = opaque(state + g);
 #pragma unroll

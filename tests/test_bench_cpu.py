@@ -94,8 +94,9 @@ def test_mickey2_deferred_reduction_op_counts():
 
 def test_mickey2_deferred_reduction_equals_galois_clocking():
     """(x + c) * R mod p clocked K times unreduced, then folded with Q_m, equals
-    K Galois clocks of the spec (r'_i = r_{i-1} ^ [i in RTAPS] r99 ^ c r_i), with
-    the taps r0 / r33 / r67 read mid-block through their pending terms."""
+    K Galois clocks of the spec (r'_i = r_{i-1} ^ [i in RTAPS] (r99 ^ u) ^ c r_i,
+    u = INPUT_BIT ^ s50 when mixing, else 0), with the taps r0 / r33 / r67 read
+    mid-block through their pending terms."""
     import random
     rng = random.Random(2020)
     taps = set(_RTAPS)
@@ -104,11 +105,13 @@ def test_mickey2_deferred_reduction_equals_galois_clocking():
         for _ in range(200):
             R = rng.getrandbits(100)
             ctl = [rng.getrandbits(1) for _ in range(k)]
+            # MIXING (initialisation): u = INPUT_BIT ^ s50 joins the feedback
+            mix = [rng.getrandbits(1) if k == 4 else 0 for _ in range(k)]
             # Galois (spec) clocks, recording r0/r33/r67 before each clock
             g, seen_g = R, []
-            for c in ctl:
+            for c, u in zip(ctl, mix):
                 seen_g.append(((g >> 0) & 1, (g >> 33) & 1, (g >> 67) & 1))
-                r99 = (g >> 99) & 1
+                r99 = ((g >> 99) & 1) ^ u
                 nxt = 0
                 for i in range(100):
                     v = ((g >> (i - 1)) & 1 if i else 0) ^ (r99 if i in taps else 0) ^ (c & (g >> i) & 1)
@@ -120,7 +123,7 @@ def test_mickey2_deferred_reduction_equals_galois_clocking():
                 pend = [(P >> (100 + m)) & 1 for m in range(j)]
                 true = lambda q: ((P >> q) & 1) ^ (sum(pend[m] & ((Q[m] >> q) & 1) for m in range(j)) & 1)
                 seen_l.append((true(0), true(33), true(67)))
-                P = (P << 1) ^ (P if c else 0)
+                P = (P << 1) ^ (P if c else 0) ^ (mix[j] << 100)  # u * x^100 == u * sum RTAPS x^t
             low = P & ((1 << 100) - 1)
             for m in range(k):
                 if (P >> (100 + m)) & 1:
