@@ -408,6 +408,84 @@ __device__ __forceinline__ uint32_t laneid_volatile()
     return v;
 }
 
+// p + d as one IMAD.WIDE.U32 (FMA pipe) instead of IADD3 + IADD3.X (ALU);
+// d < 2^32 (row strides)
+__device__ __forceinline__ uint8_t* add_fma(uint8_t* p, uint64_t d)
+{
+    uint64_t r;
+    asm("mad.wide.u32 %0, %1, 1, %2;" : "=l"(r) : "r"(uint32_t(d)), "l"(reinterpret_cast<uint64_t>(p)));
+    return reinterpret_cast<uint8_t*>(r);
+}
+
+// v[0..15] <- tcgen05.ld.16x256b.x4 at taddr: thread t receives, for repeat
+// i = 0..3 (columns +8i), TMEM lane base+t/4 columns 2(t%4), 2(t%4)+1 in
+// v[4i], v[4i+1] and lane base+8+t/4 (same columns) in v[4i+2], v[4i+3]
+// (fragment layout measured on the B200: tools/microbench/tmem_layout.cu).
+__device__ __forceinline__ void tmem_ld16x256b_x4(uint32_t taddr, uint32_t (&v)[16])
+{
+    asm volatile(
+        "tcgen05.ld.sync.aligned.16x256b.x4.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, "
+        "%15}, [%16];\n\t"
+        "tcgen05.wait::ld.sync.aligned;"
+        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+          "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
+        : "r"(taddr)
+        : "memory");
+}
+
+// Whole-sector flush (slots 0..7 of every row, 8 B aligned rows) read back
+// with the 16x256b shape: four consecutive threads receive one TMEM lane's
+// (= one instance row's) 32 B sector, so each 8 B store instruction writes 8
+// complete sectors (8 L1 wavefronts) instead of 32 half sectors from 32
+// threads' own rows (the 32x32b read-back: 2048 wavefronts and 2048 partial
+// sector writes per flush, 22% of Grain's ROW_MAJOR time in ncu's stall
+// samples).  row0s / nvalids: this warp's per-thread row bases and row counts
+// (shared memory, indexed by the thread = TMEM lane that computed them).
+__device__ __forceinline__ void rowmajor_store_tmem_sectors(uint32_t tm, uint8_t* const* row0s,
+                                                            const uint32_t* nvalids, uint64_t row_bytes, uint64_t col)
+{
+    tmem_wait_st();
+    const uint32_t t = laneid_volatile();
+#pragma unroll 1
+    for (uint32_t h = 0; h < 2; ++h) {
+        const uint32_t la = 16 * h + (t >> 2), lb = la + 8;
+        // running row pointers: 64-bit adds per row instead of multiplies
+        uint8_t* pa = row0s[la] + col + 8 * (t & 3);
+        uint8_t* pb = row0s[lb] + col + 8 * (t & 3);
+        const uint32_t na = nvalids[la], nb = nvalids[lb];
+        if (__all_sync(0xFFFFFFFFu, (na & nb) == 32)) {
+            // every row real (all but the last warp-unit): no predicates, and
+            // the row addresses advance on the FMA pipe (IMAD.WIDE) -- the
+            // clock loop saturates the ALU pipe
+#pragma unroll 1
+            for (uint32_t q0 = 0; q0 < 32; q0 += 4) {
+                uint32_t v[16];
+                tmem_ld16x256b_x4(tm + ((16 * h) << 16) + q0 * 8, v);
+#pragma unroll
+                for (int i = 0; i < 4; ++i) {
+                    __stcs(reinterpret_cast<uint2*>(pa), make_uint2(v[4 * i], v[4 * i + 1]));
+                    __stcs(reinterpret_cast<uint2*>(pb), make_uint2(v[4 * i + 2], v[4 * i + 3]));
+                    pa = add_fma(pa, row_bytes);
+                    pb = add_fma(pb, row_bytes);
+                }
+            }
+            continue;
+        }
+#pragma unroll 1
+        for (uint32_t q0 = 0; q0 < 32; q0 += 4) {
+            uint32_t v[16];
+            tmem_ld16x256b_x4(tm + ((16 * h) << 16) + q0 * 8, v);
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+                if (q0 + i < na) __stcs(reinterpret_cast<uint2*>(pa), make_uint2(v[4 * i], v[4 * i + 1]));
+                if (q0 + i < nb) __stcs(reinterpret_cast<uint2*>(pb), make_uint2(v[4 * i + 2], v[4 * i + 3]));
+                pa += row_bytes;
+                pb += row_bytes;
+            }
+        }
+    }
+}
+
 // Fetch the next work item for this warp into smem (persistent mode).
 __device__ __forceinline__ void next_item(const KsArgs& a, volatile uint32_t* slot)
 {
@@ -568,12 +646,16 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
                 if (k == NSLOT - 1 || blk + 1 == nblk) {
                     const uint32_t k_lo = k - (blk < k ? blk : k);
                     const uint32_t t = tid_volatile();
-                    if constexpr (TMEM)
-                        rowmajor_store_tmem(tm_addr(), s_row0[t], a.row_bytes, s_nvalid[t], k_lo, k,
-                                            (B - (k - k_lo)) * 4);
+                    const uint64_t col = (B - (k - k_lo)) * 4;
+                    if constexpr (TMEM) {
+                        if (k_lo == 0 && k == 7 && ((a.row_bytes | col) & 7) == 0 && a.row_bytes < (1ull << 32))
+                            rowmajor_store_tmem_sectors(tm_addr(), s_row0 + (t & ~31u), s_nvalid + (t & ~31u),
+                                                        a.row_bytes, col);
+                        else
+                            rowmajor_store_tmem(tm_addr(), s_row0[t], a.row_bytes, s_nvalid[t], k_lo, k, col);
+                    }
                     else
-                        rowmajor_store<SLOTS>(os_ptr(), s_row0[t], a.row_bytes, s_nvalid[t], k_lo, k,
-                                              (B - (k - k_lo)) * 4);
+                        rowmajor_store<SLOTS>(os_ptr(), s_row0[t], a.row_bytes, s_nvalid[t], k_lo, k, col);
                 }
             }
         }
