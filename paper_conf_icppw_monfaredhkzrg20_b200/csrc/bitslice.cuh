@@ -151,6 +151,15 @@ __device__ __forceinline__ void bt_transpose16(uint32_t (&x)[16])
 // word to put(bit, word): bit 32c+31-r (MSB) or 32c+r (LSB).  The group's
 // bytes are read with 16 B loads straight into registers (no smem staging).
 // ---------------------------------------------------------------------------
+// Where group g's 32 byte strings live: groups g < g_split straight in the
+// caller's row-major input (device inputs, no staging copy), the rest (the
+// partial last group and the padding groups) in a zero-padded tail buffer.
+__device__ __forceinline__ const uint8_t* group_src(const uint8_t* main, const uint8_t* tail, uint64_t g_split,
+                                                    uint64_t g, uint32_t group_bytes)
+{
+    return g < g_split ? main + g * group_bytes : tail + (g - g_split) * group_bytes;
+}
+
 template <int NBYTES, int NBITS, bool MSB, class Put>
 __device__ __forceinline__ void slice_group32(const uint8_t* __restrict__ p, Put&& put)
 {
@@ -207,12 +216,14 @@ __device__ __forceinline__ void slice_group32(const uint8_t* __restrict__ p, Put
 // per group; raw = Gp*32 rows of NBYTES, 16 B aligned, zero past n.
 template <int NBYTES, int NBITS, bool MSB>
 __global__ void __launch_bounds__(128) slice_state_kernel(const uint8_t* __restrict__ raw,
+                                                          const uint8_t* __restrict__ tail, uint64_t g_split,
                                                           uint32_t* __restrict__ state, uint64_t Gp)
 {
     const uint64_t g = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
     if (g >= Gp) return;
     uint32_t* p = state + g;
-    slice_group32<NBYTES, NBITS, MSB>(raw + g * (32u * NBYTES), [&](int bit, uint32_t w) { p[uint64_t(bit) * Gp] = w; });
+    slice_group32<NBYTES, NBITS, MSB>(group_src(raw, tail, g_split, g, 32u * NBYTES),
+                                      [&](int bit, uint32_t w) { p[uint64_t(bit) * Gp] = w; });
 }
 
 // Hide a pointer's provenance from the optimiser (no code emitted beyond a

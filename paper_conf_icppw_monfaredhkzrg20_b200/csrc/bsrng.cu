@@ -84,6 +84,11 @@ struct bsrng {
     uint32_t* sched = nullptr;   // [1 + units]: ticket, flags; then [32] scratch
     uint8_t* bounce = nullptr;   // generate_host staging
     uint32_t* rk_dev = nullptr;  // AES: round-key masks written by the key-expansion kernel
+    // device-input rekeys read whole 32-instance groups straight from the
+    // caller's arrays; the partial last group and the padding groups (< 32)
+    // come from this zeroed buffer: keys [32 groups * 32][key_bytes], then IVs
+    uint8_t* tail = nullptr;
+    uint64_t tail_iv_off = 0;
     bsk::aes::RoundKeys rk;      // AES: host copy, passed by value as a kernel parameter
     uint64_t bounce_bytes = 0;
     // options
@@ -128,14 +133,17 @@ int check_launch(const char* what)
     return BSRNG_OK;
 }
 
-// slice + initialisation clocks from h->raw into h->state
-int run_init(bsrng_t* h, cudaStream_t st)
+// slice + initialisation clocks into h->state.  Groups g < g_split are read
+// from raw_k / raw_iv (+ g * 32 * bytes), the rest from h->tail; the staged
+// path passes h->raw and g_split = Gp.
+int run_init(bsrng_t* h, cudaStream_t st, const uint8_t* raw_k, const uint8_t* raw_iv, uint64_t g_split)
 {
     const uint64_t kbits = uint64_t(h->key_bytes) * 8, ivbits = uint64_t(h->iv_bytes) * 8;
     uint32_t* key_s = h->sliced;
     uint32_t* iv_s = h->sliced + kbits * h->Gp;
-    const uint8_t* raw_k = h->raw;
-    const uint8_t* raw_iv = h->raw + h->iv_off;
+    const uint8_t* tail_k = h->tail;
+    const uint8_t* tail_iv = h->tail + h->tail_iv_off;
+    const bool staged = g_split >= h->Gp;
     const unsigned sblocks = unsigned((h->Gp + bsk::SLICE_GROUPS - 1) / bsk::SLICE_GROUPS);
     switch (h->cipher) {
     case BSRNG_MICKEY2: {
@@ -149,10 +157,11 @@ int run_init(bsrng_t* h, cudaStream_t st)
                 if (e != cudaSuccess) return fail(BSRNG_ECUDA, "smem attribute: %s", cudaGetErrorString(e));
                 attr = true;
             }
-            bsk::m2_init_kernel<<<blocks, bsk::M2I_BLOCK, bsk::M2I_SMEM_BYTES, st>>>(raw_k, raw_iv, int(h->iv_bits),
-                                                                                       h->state, h->Gp);
+            bsk::m2_init_kernel<<<blocks, bsk::M2I_BLOCK, bsk::M2I_SMEM_BYTES, st>>>(
+                raw_k, raw_iv, tail_k, tail_iv, g_split, int(h->iv_bits), h->state, h->Gp);
             return check_launch("m2_init");
         }
+        if (!staged) return fail(BSRNG_EINVAL, "unfused init needs staged inputs");
         bsk::slice_bits_kernel<10, 80, true><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_k, h->n, key_s, h->Gp);
         if (int rc = check_launch("slice(key)")) return rc;
         bsk::slice_bits_kernel<10, 80, true><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_iv, h->n, iv_s, h->Gp);
@@ -167,9 +176,10 @@ int run_init(bsrng_t* h, cudaStream_t st)
         // spec [15]: key and IV bits are taken LSB-first from their bytes
         if (h->opt_init_fused) {
             const unsigned blocks = unsigned((h->Gp + 127) / 128);
-            bsk::grain_init_kernel<<<blocks, 128, 0, st>>>(raw_k, raw_iv, h->state, h->Gp);
+            bsk::grain_init_kernel<<<blocks, 128, 0, st>>>(raw_k, raw_iv, tail_k, tail_iv, g_split, h->state, h->Gp);
             return check_launch("grain_init");
         }
+        if (!staged) return fail(BSRNG_EINVAL, "unfused init needs staged inputs");
         bsk::slice_bits_kernel<10, 80, false><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_k, h->n, key_s, h->Gp);
         if (int rc = check_launch("slice(key)")) return rc;
         bsk::slice_bits_kernel<8, 64, false><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_iv, h->n, iv_s, h->Gp);
@@ -182,9 +192,12 @@ int run_init(bsrng_t* h, cudaStream_t st)
         // initial counter blocks sliced straight into the state rows (FIPS-197
         // bit order: bit 0 = MSB of byte 0); round keys from the one key.
         if (h->opt_init_fused)
-            bsk::slice_state_kernel<16, 128, true><<<unsigned((h->Gp + 127) / 128), 128, 0, st>>>(raw_iv, h->state, h->Gp);
-        else
+            bsk::slice_state_kernel<16, 128, true><<<unsigned((h->Gp + 127) / 128), 128, 0, st>>>(
+                raw_iv, tail_iv, g_split, h->state, h->Gp);
+        else if (staged)
             bsk::slice_bits_kernel<16, 128, true><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_iv, h->n, h->state, h->Gp);
+        else
+            return fail(BSRNG_EINVAL, "unfused init needs staged inputs");
         if (int rc = check_launch("slice(ctr)")) return rc;
         bsk::aes::aes_key_expand_kernel<<<1, 32, 0, st>>>(raw_k, h->rk_dev);
         if (int rc = check_launch("aes_key_expand")) return rc;
@@ -200,9 +213,12 @@ int run_init(bsrng_t* h, cudaStream_t st)
     case BSRNG_LFSR128: {
         // the state IS the key: 128 bits, MSB-first, sliced straight into rows 0..127
         if (h->opt_init_fused)
-            bsk::slice_state_kernel<16, 128, true><<<unsigned((h->Gp + 127) / 128), 128, 0, st>>>(raw_k, h->state, h->Gp);
-        else
+            bsk::slice_state_kernel<16, 128, true><<<unsigned((h->Gp + 127) / 128), 128, 0, st>>>(
+                raw_k, tail_k, g_split, h->state, h->Gp);
+        else if (staged)
             bsk::slice_bits_kernel<16, 128, true><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_k, h->n, h->state, h->Gp);
+        else
+            return fail(BSRNG_EINVAL, "unfused init needs staged inputs");
         if (int rc = check_launch("slice(key)")) return rc;
         cudaError_t e = cudaMemsetAsync(h->state + uint64_t(bsk::Lfsr128::NSTATE) * h->Gp, 0, h->Gp * 4, st);
         if (e != cudaSuccess) return fail(BSRNG_ECUDA, "memset: %s", cudaGetErrorString(e));
@@ -575,14 +591,17 @@ bsrng_t* bsrng_create_ex(bsrng_cipher cipher, const uint8_t* keys, const uint8_t
         cudaMalloc(&h->sliced, sl_words * 4) != cudaSuccess ||
         cudaMalloc(&h->raw, raw_bytes) != cudaSuccess ||
         cudaMalloc(&h->sched, (1 + h->units + 32) * 4) != cudaSuccess ||
-        (aes && cudaMalloc(&h->rk_dev, sizeof(bsk::aes::RoundKeys)) != cudaSuccess)) {
+        (aes && cudaMalloc(&h->rk_dev, sizeof(bsk::aes::RoundKeys)) != cudaSuccess) ||
+        cudaMalloc(&h->tail, 32 * 32 * uint64_t(h->key_bytes + h->iv_bytes)) != cudaSuccess) {
         cudaGetLastError();
         bsrng_destroy(h);
         fail(BSRNG_ENOMEM, "cudaMalloc failed for %llu instances", (unsigned long long)n);
         return nullptr;
     }
+    h->tail_iv_off = 32 * 32 * uint64_t(h->key_bytes);
     cudaStream_t st = static_cast<cudaStream_t>(stream);
-    if (cudaMemsetAsync(h->raw, 0, raw_bytes, st) != cudaSuccess) {
+    if (cudaMemsetAsync(h->raw, 0, raw_bytes, st) != cudaSuccess ||
+        cudaMemsetAsync(h->tail, 0, 32 * 32 * uint64_t(h->key_bytes + h->iv_bytes), st) != cudaSuccess) {
         bsrng_destroy(h);
         fail(BSRNG_ECUDA, "memset(raw) failed");
         return nullptr;
@@ -616,6 +635,29 @@ int bsrng_rekey(bsrng_t* h, const uint8_t* keys, const uint8_t* ivs, uint32_t fl
     DeviceGuard dg(h->dev);
     if (!dg.ok) return fail(BSRNG_ECUDA, "cudaSetDevice(%d) failed", h->dev);
     cudaStream_t st = static_cast<cudaStream_t>(stream);
+    // Device inputs, 16 B aligned, fused init: the init kernels read whole
+    // groups straight from the caller's arrays (no staging copy, ~25 us per
+    // 2^22 keys); only the partial last group goes through h->tail.
+    const bool aes = h->cipher == BSRNG_AES128_CTR;
+    const bool direct = (flags & BSRNG_INPUT_DEVICE) && h->opt_init_fused && h->tail && ivs &&
+                        ((reinterpret_cast<uintptr_t>(keys) | reinterpret_cast<uintptr_t>(ivs)) & 15) == 0 &&
+                        !(h->cipher == BSRNG_MICKEY2 && h->iv_bytes != 10);
+    if (direct) {
+        const uint64_t g_split = h->n / 32, rest = h->n - g_split * 32;
+        cudaError_t e = cudaSuccess;
+        if (rest) {
+            if (!aes && h->key_bytes)
+                e = cudaMemcpyAsync(h->tail, keys + g_split * 32 * h->key_bytes, rest * h->key_bytes,
+                                    cudaMemcpyDeviceToDevice, st);
+            if (e == cudaSuccess && h->iv_bytes)
+                e = cudaMemcpyAsync(h->tail + h->tail_iv_off, ivs + g_split * 32 * h->iv_bytes, rest * h->iv_bytes,
+                                    cudaMemcpyDeviceToDevice, st);
+            if (e != cudaSuccess) return fail(BSRNG_ECUDA, "tail copy: %s", cudaGetErrorString(e));
+        }
+        if (int rc = run_init(h, st, keys, ivs, g_split)) return rc;
+        h->bits_done = 0;
+        return BSRNG_OK;
+    }
     if (!ivs) {  // iv_bits == 0: IV bytes are never read; keep them defined
         cudaError_t e = cudaMemsetAsync(h->raw + h->iv_off, 0, h->n * h->iv_bytes, st);
         if (e != cudaSuccess) return fail(BSRNG_ECUDA, "memset: %s", cudaGetErrorString(e));
@@ -625,7 +667,7 @@ int bsrng_rekey(bsrng_t* h, const uint8_t* keys, const uint8_t* ivs, uint32_t fl
     } else if (int rc = copy_inputs(h, keys, ivs, flags, st)) {
         return rc;
     }
-    if (int rc = run_init(h, st)) return rc;
+    if (int rc = run_init(h, st, h->raw, h->raw + h->iv_off, h->Gp)) return rc;
     h->bits_done = 0;
     return BSRNG_OK;
 }
@@ -779,6 +821,7 @@ void bsrng_destroy(bsrng_t* h)
     if (h->sched) cudaFree(h->sched);
     if (h->bounce) cudaFree(h->bounce);
     if (h->rk_dev) cudaFree(h->rk_dev);
+    if (h->tail) cudaFree(h->tail);
     delete h;
 }
 

@@ -180,17 +180,20 @@ __global__ void __launch_bounds__(128) grain_preclock_kernel(const uint32_t* __r
 // Fused slicing + initialisation (steps a-1 + a-2 in one kernel): each thread
 // slices its 32 instances' key and IV bytes in registers (slice_group32, LSB
 // first) straight into the NFSR / LFSR state words -- no sliced copy in HBM,
-// no shared memory -- then runs the 160 init clocks.  raw_k / raw_iv: regions
-// of Gp*32*10 and Gp*32*8 bytes, 16 B aligned, zero beyond instance n.
+// no shared memory -- then runs the 160 init clocks.  Group g's keys / IVs
+// at raw_k + 320 g / raw_iv + 256 g for g < g_split (16 B aligned), else in
+// the zero-padded tail buffers (see m2_init_kernel).
 __global__ void __launch_bounds__(128) grain_init_kernel(const uint8_t* __restrict__ raw_k,
                                                          const uint8_t* __restrict__ raw_iv,
+                                                         const uint8_t* __restrict__ tail_k,
+                                                         const uint8_t* __restrict__ tail_iv, uint64_t g_split,
                                                          uint32_t* __restrict__ state, uint64_t Gp)
 {
     const uint64_t g = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
     if (g >= Gp) return;
     uint32_t s[80], b[80];
-    slice_group32<10, 80, false>(raw_k + g * 320u, [&](int bit, uint32_t w) { b[bit] = w; });
-    slice_group32<8, 64, false>(raw_iv + g * 256u, [&](int bit, uint32_t w) { s[bit] = w; });
+    slice_group32<10, 80, false>(group_src(raw_k, tail_k, g_split, g, 320u), [&](int bit, uint32_t w) { b[bit] = w; });
+    slice_group32<8, 64, false>(group_src(raw_iv, tail_iv, g_split, g, 256u), [&](int bit, uint32_t w) { s[bit] = w; });
 #pragma unroll
     for (int i = 64; i < 80; ++i) s[i] = 0xFFFFFFFFu;
 #pragma unroll 1

@@ -441,22 +441,27 @@ namespace bsk {
 // pressure), and parks the 160 slice words in shared memory [bit][thread];
 // the 260 mixing clocks then read their input word from shared memory.
 // 20 KB of smem per warp -> two 4-warp CTAs (two warps per SMSP) per SM.
-// Inputs: raw_k / raw_iv regions of Gp*32*10 bytes, 16 B aligned, zero
-// beyond instance n (bsrng.cu allocates and zero-fills them).
+// Inputs: group g's 32 keys / IVs (10 B each) at raw_k / raw_iv + 320 g for
+// g < g_split (16 B aligned; the caller's device arrays or the staging copy),
+// else at tail_k / tail_iv + 320 (g - g_split) (zero beyond instance n).
 // ---------------------------------------------------------------------------
 constexpr int M2I_BLOCK = 128;
 constexpr size_t M2I_SMEM_BYTES = size_t(160) * M2I_BLOCK * 4;  // [IV bit 0..79, key bit 0..79][thread]
 
 __global__ void __launch_bounds__(M2I_BLOCK, 2) m2_init_kernel(const uint8_t* __restrict__ raw_k,
-                                                              const uint8_t* __restrict__ raw_iv, int iv_bits,
-                                                              uint32_t* __restrict__ state, uint64_t Gp)
+                                                              const uint8_t* __restrict__ raw_iv,
+                                                              const uint8_t* __restrict__ tail_k,
+                                                              const uint8_t* __restrict__ tail_iv, uint64_t g_split,
+                                                              int iv_bits, uint32_t* __restrict__ state, uint64_t Gp)
 {
     extern __shared__ uint32_t m2i_smem[];
     const uint64_t g = uint64_t(blockIdx.x) * M2I_BLOCK + threadIdx.x;
     if (g >= Gp) return;  // no block-level barrier below
     uint32_t* sl = m2i_smem + threadIdx.x;
-    slice_group32<10, 80, true>(raw_iv + g * 320u, [&](int bit, uint32_t w) { sl[bit * M2I_BLOCK] = w; });
-    slice_group32<10, 80, true>(raw_k + g * 320u, [&](int bit, uint32_t w) { sl[(80 + bit) * M2I_BLOCK] = w; });
+    slice_group32<10, 80, true>(group_src(raw_iv, tail_iv, g_split, g, 320u),
+                                [&](int bit, uint32_t w) { sl[bit * M2I_BLOCK] = w; });
+    slice_group32<10, 80, true>(group_src(raw_k, tail_k, g_split, g, 320u),
+                                [&](int bit, uint32_t w) { sl[(80 + bit) * M2I_BLOCK] = w; });
 
     // R with the deferred reduction (m2::clock_lazy, 4-clock blocks; reduced
     // again at every block boundary, so the stored state is the spec's)
