@@ -27,12 +27,13 @@ cap() {
   rm -f /tmp/prof_$name.ncu-rep
 }
 cap ks_consume keystream_kernel python tools/prof_driver.py --layout checksum --bits 65536 --reps 2
-cap ks_rowmajor rm_ws python tools/prof_driver.py --layout row_major --bits 32768 --reps 2
+cap ks_rowmajor keystream_kernel python tools/prof_driver.py --layout row_major --bits 32768 --reps 2
 cap ks_sliced keystream_kernel python tools/prof_driver.py --layout sliced --bits 4096 --reps 2
 cap grain_consume keystream_kernel python tools/prof_driver.py --cipher grain --layout checksum --bits 65536 --reps 2
 cap grain_rowmajor keystream_kernel python tools/prof_driver.py --cipher grain --layout row_major --bits 32768 --reps 2
 cap aes_consume aes_ctr python tools/prof_driver.py --cipher aes128ctr --layout checksum --bits 16384 --reps 2
 cap aes_rowmajor rowmajor_lanes python tools/prof_driver.py --cipher aes128ctr --layout row_major --bits 16384 --reps 2
 cap lfsr_sliced keystream_kernel python tools/prof_driver.py --cipher lfsr128 --layout sliced --bits 65536 --reps 2
-cap preclock m2_preclock python tools/prof_driver.py --layout checksum --bits 32 --reps 1
+cap preclock m2_init python tools/prof_driver.py --layout checksum --bits 32 --reps 1
+cap grain_init grain_init python tools/prof_driver.py --cipher grain --layout checksum --bits 32 --reps 1
 ls -la gpurun_out/prof gpurun_out/bench
