@@ -168,6 +168,34 @@ def profile_traffic():
         return None
 
 
+# committed ncu --set full capture (tools/gpu_profile.sh) per cipher and mode
+TRAFFIC_CAPTURE = {("mickey2", "consume"): "ks_consume", ("mickey2", "materialise"): "ks_rowmajor",
+                   ("grain", "consume"): "grain_consume", ("grain", "materialise"): "grain_rowmajor",
+                   ("aes128ctr", "consume"): "aes_consume", ("aes128ctr", "materialise"): "aes_rowmajor",
+                   ("lfsr128", "materialise"): "lfsr_sliced"}
+
+
+def traffic_for(cipher, mode, n, launch_bits):
+    """(dram read + write bytes per launch, note) for the dominant kernel from
+    the committed capture of the same kernel at n instances.  Consume launches
+    move only the state carry (same per launch at any bit count); materialise
+    writes scale with the bits per launch, so the capture's write bytes are
+    scaled by launch_bits / captured bits when the two differ."""
+    tr = profile_traffic()
+    cap = (tr or {}).get("captures", {}).get(TRAFFIC_CAPTURE.get((cipher, mode), ""))
+    if not cap or f"n={n}" not in cap.get("driver", ""):
+        return None, None
+    import re
+    m = re.search(r"bits=(\d+)", cap.get("driver", ""))
+    cap_bits = int(m.group(1)) if m else None
+    rd, wr = cap["dram_read"], cap["dram_write"]
+    note = f"ncu --set full capture '{TRAFFIC_CAPTURE[(cipher, mode)]}' (profiles/, n={n}, {cap_bits} bits per launch)"
+    if mode == "materialise" and cap_bits and cap_bits != launch_bits:
+        wr *= launch_bits / cap_bits
+        note += f"; writes scaled to {launch_bits} bits per launch"
+    return rd + wr, note
+
+
 def cpu_cores():
     try:
         return len(os.sched_getaffinity(0))
@@ -482,10 +510,12 @@ def run_ours(args, rank, world, local_rank):
     if rank == 0:
         head = results[args.mode]
         rf = head["roofline"]
-        tr = profile_traffic()
-        if tr and tr.get("mode") == args.mode and tr.get("n") == n:
-            rf["traffic"] = tr.get("dram_bytes_per_launch")
-            rf["traffic_note"] = tr.get("note")
+        for mode, res in results.items():
+            lb = bits if mode == "consume" else min(bits, args.chunk_bits)
+            t, note = traffic_for(args.cipher, mode, n, lb)
+            if t is not None:
+                res["roofline"]["traffic"] = t
+                res["roofline"]["traffic_note"] = note
         line = {
             "metric": metric(args), "value": head["value"], "unit": "Tb/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": head["ms_per_step"],
