@@ -21,7 +21,7 @@ ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpuru
 # each, over gpurun's 64 MiB copy-back limit) and the reports deleted
 cap() {
   name=$1; shift
-  ncu --set full --clock-control none --import-source on -k regex:$1 -s 1 -c 1 -o /tmp/prof_$name "${@:2}" > gpurun_out/prof/ncu_$name.log 2>&1
+  ncu --set full --clock-control none --import-source on -k regex:$1 -s ${SKIP:-1} -c 1 -o /tmp/prof_$name "${@:2}" > gpurun_out/prof/ncu_$name.log 2>&1
   ncu -i /tmp/prof_$name.ncu-rep --page raw --csv > gpurun_out/prof/${name}_raw.csv 2>/dev/null
   ncu -i /tmp/prof_$name.ncu-rep --page details --csv > gpurun_out/prof/${name}_details.csv 2>/dev/null
   rm -f /tmp/prof_$name.ncu-rep
@@ -34,6 +34,6 @@ cap grain_rowmajor keystream_kernel python tools/prof_driver.py --cipher grain -
 cap aes_consume aes_ctr python tools/prof_driver.py --cipher aes128ctr --layout checksum --bits 16384 --reps 2
 cap aes_rowmajor rowmajor_lanes python tools/prof_driver.py --cipher aes128ctr --layout row_major --bits 16384 --reps 2
 cap lfsr_sliced keystream_kernel python tools/prof_driver.py --cipher lfsr128 --layout sliced --bits 65536 --reps 2
-cap preclock m2_init python tools/prof_driver.py --layout checksum --bits 32 --reps 1
-cap grain_init grain_init python tools/prof_driver.py --cipher grain --layout checksum --bits 32 --reps 1
+SKIP=0 cap preclock m2_init python tools/prof_driver.py --layout checksum --bits 32 --reps 1
+SKIP=0 cap grain_init grain_init python tools/prof_driver.py --cipher grain --layout checksum --bits 32 --reps 1
 ls -la gpurun_out/prof gpurun_out/bench
