@@ -89,7 +89,12 @@ def point(cipher, n, bits, layout, opts, reps, chunk=None, nsm=148):
     del out
     mhz = cs.median() or 1965
     tbps = n * bits / (best * 1e-3) / 1e12
-    ops = OPS[cipher] * (n / 32) * bits / (best * 1e-3)
+    per_clock = OPS[cipher]
+    if cipher == "mickey2" and "unroll" in opts:  # deferred-reduction block K follows U (bench.py)
+        sys.path.insert(0, ROOT)
+        import bench
+        per_clock = bench.lop3_per_bit("mickey2", "consume", opts["unroll"])
+    ops = per_clock * (n / 32) * bits / (best * 1e-3)
     peak = nsm * 64 * mhz * 1e6
     return {"cipher": cipher, "n": n, "clocks_per_call": chunk, "clocks": bits, "layout": layout, "opts": opts,
             "ms": round(best, 3), "tbps": round(tbps, 4), "sm_mhz": mhz, "alu_frac": round(ops / peak, 4)}
