@@ -160,7 +160,37 @@ __device__ __forceinline__ const uint8_t* group_src(const uint8_t* main, const u
     return g < g_split ? main + g * group_bytes : tail + (g - g_split) * group_bytes;
 }
 
-template <int NBYTES, int NBITS, bool MSB, class Put>
+// Stage a warp's 32 consecutive group blocks (GB bytes each, contiguous in
+// global memory from `src`) into shared memory, one row of STRIDE bytes per
+// lane, with coalesced 16 B loads (512 contiguous bytes per instruction).
+// Per-thread 16 B loads of the own 320 B block touch 32 lines per instruction
+// (8x the L1 wavefronts); ncu: long-scoreboard stalls at 0.31 per issue in
+// the Grain init kernel.  STRIDE = GB + 16 keeps the lanes' 16 B smem reads
+// of their own rows bank-conflict free.
+template <int GB, int STRIDE>
+__device__ __forceinline__ void stage_warp_groups(const uint8_t* __restrict__ src, uint8_t* dst, uint32_t lane)
+{
+    static_assert(GB % 16 == 0 && STRIDE % 16 == 0, "16 B pieces");
+    constexpr int PIECES = GB / 16;
+    const uint4* s = reinterpret_cast<const uint4*>(src);
+#pragma unroll
+    for (int k = 0; k < PIECES; ++k) {
+        const uint32_t P = lane + 32u * k;
+        const uint4 v = __ldcs(s + P);
+        *reinterpret_cast<uint4*>(dst + (P / PIECES) * STRIDE + (P % PIECES) * 16) = v;
+    }
+}
+// The same for one lane's own block (warps whose groups are not contiguous).
+template <int GB, int STRIDE>
+__device__ __forceinline__ void stage_own_group(const uint8_t* __restrict__ src, uint8_t* dst, uint32_t lane)
+{
+    const uint4* s = reinterpret_cast<const uint4*>(src);
+#pragma unroll
+    for (int k = 0; k < GB / 16; ++k) *reinterpret_cast<uint4*>(dst + lane * STRIDE + 16 * k) = __ldcs(s + k);
+}
+
+// GLOBAL: p is global memory (streaming 16 B loads); else shared memory.
+template <int NBYTES, int NBITS, bool MSB, bool GLOBAL = true, class Put>
 __device__ __forceinline__ void slice_group32(const uint8_t* __restrict__ p, Put&& put)
 {
     static_assert((32 * NBYTES) % 16 == 0, "group block must be whole 16 B vectors");
@@ -169,7 +199,7 @@ __device__ __forceinline__ void slice_group32(const uint8_t* __restrict__ p, Put
     const uint4* src = reinterpret_cast<const uint4*>(p);
 #pragma unroll
     for (int i = 0; i < NW / 4; ++i) {
-        const uint4 v = __ldcs(src + i);
+        const uint4 v = GLOBAL ? __ldcs(src + i) : src[i];
         raw[4 * i] = v.x;
         raw[4 * i + 1] = v.y;
         raw[4 * i + 2] = v.z;
@@ -214,16 +244,30 @@ __device__ __forceinline__ void slice_group32(const uint8_t* __restrict__ p, Put
 // Slice 32-instance group blocks straight into state rows [bit][Gp] (AES-CTR
 // initial counters, LFSR keys: the sliced input IS the state).  One thread
 // per group; raw = Gp*32 rows of NBYTES, 16 B aligned, zero past n.
+// The warp's group blocks are staged through shared memory with coalesced
+// loads (stage_warp_groups); SS_SMEM_BYTES(NBYTES) of dynamic smem per CTA.
+__host__ __device__ constexpr int ss_stride(int nbytes) { return 32 * nbytes + 16; }
+__host__ __device__ constexpr size_t ss_smem_bytes(int nbytes) { return size_t(128) * ss_stride(nbytes); }
+
 template <int NBYTES, int NBITS, bool MSB>
 __global__ void __launch_bounds__(128) slice_state_kernel(const uint8_t* __restrict__ raw,
                                                           const uint8_t* __restrict__ tail, uint64_t g_split,
                                                           uint32_t* __restrict__ state, uint64_t Gp)
 {
+    constexpr int GB = 32 * NBYTES, STRIDE = ss_stride(NBYTES);
+    extern __shared__ __align__(16) uint8_t ss_smem[];
     const uint64_t g = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
-    if (g >= Gp) return;
+    if (g >= Gp) return;  // whole warps (Gp is a multiple of 32)
+    const uint32_t lane = threadIdx.x & 31u;
+    uint8_t* w = ss_smem + (threadIdx.x >> 5) * 32 * STRIDE;
+    const uint64_t g0 = g - lane;
+    if (g0 + 32 <= g_split)
+        stage_warp_groups<GB, STRIDE>(raw + g0 * GB, w, lane);
+    else
+        stage_own_group<GB, STRIDE>(group_src(raw, tail, g_split, g, GB), w, lane);
+    __syncwarp();
     uint32_t* p = state + g;
-    slice_group32<NBYTES, NBITS, MSB>(group_src(raw, tail, g_split, g, 32u * NBYTES),
-                                      [&](int bit, uint32_t w) { p[uint64_t(bit) * Gp] = w; });
+    slice_group32<NBYTES, NBITS, MSB, false>(w + lane * STRIDE, [&](int bit, uint32_t v) { p[uint64_t(bit) * Gp] = v; });
 }
 
 // Hide a pointer's provenance from the optimiser (no code emitted beyond a

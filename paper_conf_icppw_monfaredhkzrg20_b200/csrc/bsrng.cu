@@ -138,6 +138,13 @@ int check_launch(const char* what)
 // path passes h->raw and g_split = Gp.
 int run_init(bsrng_t* h, cudaStream_t st, const uint8_t* raw_k, const uint8_t* raw_iv, uint64_t g_split)
 {
+    static bool ss_attr = false;  // > 48 KB of dynamic smem (coalesced staging)
+    if (!ss_attr) {
+        cudaError_t e = cudaFuncSetAttribute(bsk::slice_state_kernel<16, 128, true>,
+                                             cudaFuncAttributeMaxDynamicSharedMemorySize, int(bsk::ss_smem_bytes(16)));
+        if (e != cudaSuccess) return fail(BSRNG_ECUDA, "smem attribute: %s", cudaGetErrorString(e));
+        ss_attr = true;
+    }
     const uint64_t kbits = uint64_t(h->key_bytes) * 8, ivbits = uint64_t(h->iv_bytes) * 8;
     uint32_t* key_s = h->sliced;
     uint32_t* iv_s = h->sliced + kbits * h->Gp;
@@ -176,7 +183,15 @@ int run_init(bsrng_t* h, cudaStream_t st, const uint8_t* raw_k, const uint8_t* r
         // spec [15]: key and IV bits are taken LSB-first from their bytes
         if (h->opt_init_fused) {
             const unsigned blocks = unsigned((h->Gp + 127) / 128);
-            bsk::grain_init_kernel<<<blocks, 128, 0, st>>>(raw_k, raw_iv, tail_k, tail_iv, g_split, h->state, h->Gp);
+            static bool gattr = false;
+            if (!gattr) {
+                cudaError_t e = cudaFuncSetAttribute(bsk::grain_init_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                     int(bsk::GI_SMEM_BYTES));
+                if (e != cudaSuccess) return fail(BSRNG_ECUDA, "smem attribute: %s", cudaGetErrorString(e));
+                gattr = true;
+            }
+            bsk::grain_init_kernel<<<blocks, 128, bsk::GI_SMEM_BYTES, st>>>(raw_k, raw_iv, tail_k, tail_iv, g_split,
+                                                                           h->state, h->Gp);
             return check_launch("grain_init");
         }
         if (!staged) return fail(BSRNG_EINVAL, "unfused init needs staged inputs");
@@ -192,7 +207,7 @@ int run_init(bsrng_t* h, cudaStream_t st, const uint8_t* raw_k, const uint8_t* r
         // initial counter blocks sliced straight into the state rows (FIPS-197
         // bit order: bit 0 = MSB of byte 0); round keys from the one key.
         if (h->opt_init_fused)
-            bsk::slice_state_kernel<16, 128, true><<<unsigned((h->Gp + 127) / 128), 128, 0, st>>>(
+            bsk::slice_state_kernel<16, 128, true><<<unsigned((h->Gp + 127) / 128), 128, bsk::ss_smem_bytes(16), st>>>(
                 raw_iv, tail_iv, g_split, h->state, h->Gp);
         else if (staged)
             bsk::slice_bits_kernel<16, 128, true><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_iv, h->n, h->state, h->Gp);
@@ -213,7 +228,7 @@ int run_init(bsrng_t* h, cudaStream_t st, const uint8_t* raw_k, const uint8_t* r
     case BSRNG_LFSR128: {
         // the state IS the key: 128 bits, MSB-first, sliced straight into rows 0..127
         if (h->opt_init_fused)
-            bsk::slice_state_kernel<16, 128, true><<<unsigned((h->Gp + 127) / 128), 128, 0, st>>>(
+            bsk::slice_state_kernel<16, 128, true><<<unsigned((h->Gp + 127) / 128), 128, bsk::ss_smem_bytes(16), st>>>(
                 raw_k, tail_k, g_split, h->state, h->Gp);
         else if (staged)
             bsk::slice_bits_kernel<16, 128, true><<<sblocks, bsk::SLICE_BLOCK, 0, st>>>(raw_k, h->n, h->state, h->Gp);

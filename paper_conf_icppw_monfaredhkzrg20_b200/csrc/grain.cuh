@@ -183,17 +183,34 @@ __global__ void __launch_bounds__(128) grain_preclock_kernel(const uint32_t* __r
 // no shared memory -- then runs the 160 init clocks.  Group g's keys / IVs
 // at raw_k + 320 g / raw_iv + 256 g for g < g_split (16 B aligned), else in
 // the zero-padded tail buffers (see m2_init_kernel).
+// key / IV rows of the shared-memory staging area (bytes per lane)
+constexpr int GI_KSTRIDE = 336, GI_VSTRIDE = 272;
+constexpr size_t GI_SMEM_BYTES = size_t(128) * (GI_KSTRIDE + GI_VSTRIDE);  // 76 KB per 4-warp CTA
+
 __global__ void __launch_bounds__(128) grain_init_kernel(const uint8_t* __restrict__ raw_k,
                                                          const uint8_t* __restrict__ raw_iv,
                                                          const uint8_t* __restrict__ tail_k,
                                                          const uint8_t* __restrict__ tail_iv, uint64_t g_split,
                                                          uint32_t* __restrict__ state, uint64_t Gp)
 {
+    extern __shared__ __align__(16) uint8_t gi_smem[];
     const uint64_t g = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
-    if (g >= Gp) return;
+    if (g >= Gp) return;  // whole warps (Gp is a multiple of 32)
+    const uint32_t lane = threadIdx.x & 31u;
+    uint8_t* wk = gi_smem + (threadIdx.x >> 5) * 32 * (GI_KSTRIDE + GI_VSTRIDE);
+    uint8_t* wv = wk + 32 * GI_KSTRIDE;
+    const uint64_t g0 = g - lane;
+    if (g0 + 32 <= g_split) {  // warp-uniform: the warp's 32 groups are contiguous
+        stage_warp_groups<320, GI_KSTRIDE>(raw_k + g0 * 320u, wk, lane);
+        stage_warp_groups<256, GI_VSTRIDE>(raw_iv + g0 * 256u, wv, lane);
+    } else {
+        stage_own_group<320, GI_KSTRIDE>(group_src(raw_k, tail_k, g_split, g, 320u), wk, lane);
+        stage_own_group<256, GI_VSTRIDE>(group_src(raw_iv, tail_iv, g_split, g, 256u), wv, lane);
+    }
+    __syncwarp();
     uint32_t s[80], b[80];
-    slice_group32<10, 80, false>(group_src(raw_k, tail_k, g_split, g, 320u), [&](int bit, uint32_t w) { b[bit] = w; });
-    slice_group32<8, 64, false>(group_src(raw_iv, tail_iv, g_split, g, 256u), [&](int bit, uint32_t w) { s[bit] = w; });
+    slice_group32<10, 80, false, false>(wk + lane * GI_KSTRIDE, [&](int bit, uint32_t w) { b[bit] = w; });
+    slice_group32<8, 64, false, false>(wv + lane * GI_VSTRIDE, [&](int bit, uint32_t w) { s[bit] = w; });
 #pragma unroll
     for (int i = 64; i < 80; ++i) s[i] = 0xFFFFFFFFu;
 #pragma unroll 1
