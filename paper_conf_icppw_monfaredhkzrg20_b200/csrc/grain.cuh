@@ -185,6 +185,9 @@ __global__ void __launch_bounds__(128) grain_preclock_kernel(const uint32_t* __r
 // the zero-padded tail buffers (see m2_init_kernel).
 // key / IV rows of the shared-memory staging area (bytes per lane)
 constexpr int GI_KSTRIDE = 336, GI_VSTRIDE = 272;
+#ifndef GI_UNROLL
+#define GI_UNROLL 40
+#endif
 constexpr size_t GI_SMEM_BYTES = size_t(128) * (GI_KSTRIDE + GI_VSTRIDE);  // 76 KB per 4-warp CTA
 
 __global__ void __launch_bounds__(128) grain_init_kernel(const uint8_t* __restrict__ raw_k,
@@ -214,9 +217,11 @@ __global__ void __launch_bounds__(128) grain_init_kernel(const uint8_t* __restri
 #pragma unroll
     for (int i = 64; i < 80; ++i) s[i] = 0xFFFFFFFFu;
 #pragma unroll 1
-    for (int c = 0; c < 160; c += 16) {
+    // 40 clocks per iteration: the 80-word rotation closes with 160 moves per
+    // 40 clocks (4 per clock on the FMA pipe; 10 at 16 clocks per iteration)
+    for (int c = 0; c < 160; c += GI_UNROLL) {
 #pragma unroll
-        for (int u = 0; u < 16; ++u) grain::clock<true>(s, b);
+        for (int u = 0; u < GI_UNROLL; ++u) grain::clock<true>(s, b);
     }
     uint32_t* p = opaque(state + g);
 #pragma unroll
