@@ -196,6 +196,16 @@ def traffic_for(cipher, mode, n, launch_bits):
     return rd + wr, note
 
 
+def state_words(cipher):
+    """sliced state rows per 32-instance group (+1 checksum row)"""
+    return {"mickey2": 201, "grain": 161, "aes128ctr": 129, "lfsr128": 129}[cipher]
+
+
+def key_iv_bytes(cipher):
+    """device-resident key/IV (counter) bytes per instance read by a rekey"""
+    return {"mickey2": 20, "grain": 18, "aes128ctr": 16, "lfsr128": 16}[cipher]
+
+
 def cpu_cores():
     try:
         return len(os.sched_getaffinity(0))
@@ -524,7 +534,9 @@ def run_ours(args, rank, world, local_rank):
             "config": {"workload": f"{desc} ({args.mode})", "instances_total": n_total,
                        "instances_per_gpu": n, "bits_per_instance": bits,
                        "mode": args.mode, "parallelism": f"instance-range shards x{world}",
-                       "l2": "flushed (256 MiB write) between timed steps; state 100 MiB, keys 80 MiB"},
+                       "l2": (f"flushed (256 MiB write) between timed steps; state "
+                              f"{state_words(args.cipher) * (n // 32) * 4 / 2**20:.0f} MiB, keys/IVs "
+                              f"{n * key_iv_bytes(args.cipher) / 2**20:.0f} MiB")},
             "roofline": rf, "clocks": head.get("clocks"), "gpu_launches": head["gpu_launches"],
             "e2e": e2e, "cpu_baseline": cpu, "checksum": f"{checksum:016x}", "context": context,
             "modes": {m: {k: v for k, v in r.items() if k != "clocks"} for m, r in results.items()},
