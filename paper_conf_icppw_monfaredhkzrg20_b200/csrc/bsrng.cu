@@ -107,6 +107,9 @@ struct bsrng {
     int opt_rm_zreg = 1;
     // ROW_MAJOR plain kernel: stage row segments in TMEM (1) or smem (0).
     int opt_rm_tmem = -1;  // -1 = the cipher's default (C::RM_TMEM)
+    // TMEM-staged ROW_MAJOR: whole-sector flushes as TMA tensor stores (1) or
+    // as 8 B global stores from the 16x256b read-back (0)
+    int opt_rm_tma = 1;
     // init: slicing fused into the init kernel (MICKEY, Grain) / per-thread group
     // slicing into the state (AES, LFSR) (1), or the ballot slice kernels (0).
     int opt_init_fused = 1;
@@ -255,6 +258,35 @@ int copy_inputs(bsrng_t* h, const uint8_t* keys, const uint8_t* ivs, uint32_t fl
     return BSRNG_OK;
 }
 
+// Tensor map for TMA ROW_MAJOR flushes (keystream.cuh rowmajor_store_tmem_tma):
+// element (byte c, group g, q) of the 3-D view = out[(32 g + q) * row_bytes + c],
+// dims {row_bytes, groups, 32}, box {32 B, 8 groups, 32}.  The driver's
+// cuTensorMapEncodeTiled is reached through the runtime's entry-point query
+// (no libcuda link dependency).
+using EncodeTiledFn = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+int encode_rowmajor_tmap(CUtensorMap* map, void* out, uint64_t row_bytes, uint64_t groups)
+{
+    static EncodeTiledFn encode = nullptr;
+    if (!encode) {
+        void* fn = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess ||
+            q != cudaDriverEntryPointSuccess || !fn)
+            return fail(BSRNG_ECUDA, "cuTensorMapEncodeTiled unavailable");
+        encode = reinterpret_cast<EncodeTiledFn>(fn);
+    }
+    const cuuint64_t dims[3] = {row_bytes, groups, 32};
+    const cuuint64_t strides[2] = {32 * row_bytes, row_bytes};
+    const cuuint32_t box[3] = {32, 8, 32}, estr[3] = {1, 1, 1};
+    const CUresult r = encode(map, CU_TENSOR_MAP_DATA_TYPE_UINT8, 3, out, dims, strides, box, estr,
+                              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                              CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return fail(BSRNG_ECUDA, "cuTensorMapEncodeTiled failed (%d)", int(r));
+    return BSRNG_OK;
+}
+
 // Kernel instance for the handle's unroll option and ROW_MAJOR staging slots.
 template <class C, int LAYOUT, int SLOTS, bool ZREG = true, bool TMEM = false>
 auto pick_keystream_kernel(const bsrng_t* h, int* U)
@@ -314,6 +346,14 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
     int block = KS_BLOCK, compute_warps = KS_BLOCK / 32;
     size_t smem = LAYOUT == bsk::L_ROW_MAJOR ? size_t(KS_BLOCK / 32) * bsk::rm_warp_words(U, slots, zreg) * 4 : 0;
     if (tmem) smem = (U == 32 && zreg) ? 0 : size_t(KS_BLOCK / 32) * bsk::ZS_WORDS * 4;
+    // TMA tensor stores for the whole-sector flushes of all-real warps: needs
+    // 16 B aligned row strides (TMA global strides) and at least one such warp
+    if (tmem && h->opt_rm_tma && (a.row_bytes % 16) == 0 && h->n / 32 >= 32 && a.row_bytes < (1ull << 32)) {
+        if (int rc = encode_rowmajor_tmap(&a.tmap, out, a.row_bytes, h->n / 32)) return rc;
+        a.use_tma = 1;
+        a.tma_groups = h->n / 32;
+        smem += size_t(KS_BLOCK / 32) * bsk::TMA_BUF_WORDS * 4;
+    }
     if (ws) {
         kern = &bsk::keystream_rm_ws_kernel<C, C::U_DEFAULT>;
         if (h->opt_unroll == C::U_ALT0) kern = &bsk::keystream_rm_ws_kernel<C, C::U_ALT0>;
@@ -812,6 +852,8 @@ int bsrng_set_option(bsrng_t* h, const char* key, int64_t value)
     } else if (!strcmp(key, "rm_zreg")) {
         if (value != 0 && value != 1) return fail(BSRNG_EINVAL, "rm_zreg must be 0 or 1");
         h->opt_rm_zreg = int(value);
+    } else if (!strcmp(key, "rm_tma")) {
+        h->opt_rm_tma = int(value);
     } else if (!strcmp(key, "rm_tmem")) {
         if (value < -1 || value > 1) return fail(BSRNG_EINVAL, "rm_tmem must be -1 (auto), 0 or 1");
         h->opt_rm_tmem = int(value);

@@ -26,6 +26,8 @@
 //              two 16-row halves to bound register pressure) and writes one
 //              32-bit word per instance row.
 #pragma once
+#include <cuda.h>  // CUtensorMap (type only; encoded on the host via the runtime's driver entry point)
+
 #include <cstdint>
 #include <type_traits>
 #include <utility>
@@ -108,6 +110,11 @@ struct KsArgs {
     const void* aux;      // cipher-specific input (AES block-lane ROW_MAJOR: counters)
     unsigned long long* dbg;  // optional scheduler counters (BSRNG_DEBUG), or null
     int persistent;
+    // ROW_MAJOR + TMEM: whole-sector flushes of warps whose 32 groups are all
+    // real (g < tma_groups) go out as TMA tensor stores (rowmajor_store_tmem_tma)
+    int use_tma;
+    uint64_t tma_groups;
+    CUtensorMap tmap;  // 3-D view of `out`: [q 32][group][byte], see bsrng.cu
 };
 
 __device__ __forceinline__ uint32_t ld_acquire(const uint32_t* p)
@@ -486,6 +493,71 @@ __device__ __forceinline__ void rowmajor_store_tmem_sectors(uint32_t tm, uint8_t
     }
 }
 
+// ---------------------------------------------------------------------------
+// TMA-store flush (ROW_MAJOR, TMEM staging).  The 16x256b read-back gives four
+// threads one row's 32 B sector; instead of 128 scattered 8 B global stores
+// per thread (whose address/data registers the next instructions must wait
+// to reuse until the LSU has drained them -- ncu: long-scoreboard stalls on
+// the flush's address adds, 12.6% of Grain's ROW_MAJOR time), each warp
+// writes the sectors into a 16 KB shared-memory box and one lane issues TMA
+// tensor stores, which move the 1024 scattered sectors asynchronously while
+// the warp returns to its clock loop.
+// Tensor map (bsrng.cu): dims {row_bytes, tma_groups, 32} with strides
+// {32 row_bytes, row_bytes}, i.e. element (byte c, group g, q) = out[(32 g + q)
+// * row_bytes + c]; box {32, 8, 32} = 8 groups x 32 instances x one 32 B
+// sector, laid out in smem as [q][group][32 B] so a 16x256b fragment (8
+// groups x 32 B for one q) is 256 contiguous bytes: conflict-free 8 B stores.
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ uint32_t smem_addr_u32(const void* p)
+{
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void bulk_wait_read_all() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void tma_store_3d(const CUtensorMap* map, uint32_t src, int c0, int c1, int c2)
+{
+    asm volatile("cp.async.bulk.tensor.3d.global.shared::cta.bulk_group [%0, {%2, %3, %4}], [%1];" ::"l"(
+                     reinterpret_cast<uint64_t>(map)),
+                 "r"(src), "r"(c0), "r"(c1), "r"(c2)
+                 : "memory");
+}
+constexpr int TMA_BUF_WORDS = 4096;  // 16 KB per warp: two 8 KB boxes
+
+__device__ __forceinline__ void rowmajor_store_tmem_tma(uint32_t tm, uint32_t* buf, const CUtensorMap* map,
+                                                        uint64_t g_w0, uint64_t col)
+{
+    tmem_wait_st();
+    const uint32_t t = laneid_volatile();
+    const uint32_t sb = smem_addr_u32(buf);
+    const uint32_t off_t = (t >> 2) * 32 + (t & 3) * 8;
+#pragma unroll 1
+    for (uint32_t h = 0; h < 2; ++h) {
+        // the previous TMA stores must have read the buffer
+        if (t == 0) bulk_wait_read_all();
+        __syncwarp();
+#pragma unroll 1
+        for (uint32_t q0 = 0; q0 < 32; q0 += 4) {
+            uint32_t v[16];
+            tmem_ld16x256b_x4(tm + ((16 * h) << 16) + q0 * 8, v);
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+                const uint32_t o = sb + (q0 + i) * 256 + off_t;
+                asm volatile("st.shared.v2.b32 [%0], {%1, %2};" ::"r"(o), "r"(v[4 * i]), "r"(v[4 * i + 1]) : "memory");
+                asm volatile("st.shared.v2.b32 [%0], {%1, %2};" ::"r"(o + 8192), "r"(v[4 * i + 2]), "r"(v[4 * i + 3])
+                             : "memory");
+            }
+        }
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic-proxy writes -> TMA reads
+        __syncwarp();
+        if (t == 0) {
+            const int g = int(g_w0 + 16 * h);
+            tma_store_3d(map, sb, int(col), g, 0);
+            tma_store_3d(map, sb + 8192, int(col), g + 8, 0);
+            asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        }
+    }
+}
+
 // Fetch the next work item for this warp into smem (persistent mode).
 __device__ __forceinline__ void next_item(const KsArgs& a, volatile uint32_t* slot)
 {
@@ -497,13 +569,15 @@ __device__ __forceinline__ void next_item(const KsArgs& a, volatile uint32_t* sl
 // SLOTS: row-segment slots staged in smem (8 or 4); TMEM: stage in tensor
 // memory instead (8 slots, no smem for rows); ZREG: see rm_warp_words.
 template <class C, int LAYOUT, int U, int BLOCK, int SLOTS = 8, bool ZREG = true, bool TMEM = false>
-__global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
+__global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant__ KsArgs a)
 {
     static_assert(32 % U == 0, "U must divide 32");
     constexpr int KB = ks_block<C, U>();  // clocks per cipher schedule block
     static_assert(U % KB == 0, "the loop body must hold whole schedule blocks");
     constexpr int NW = BLOCK / 32;
-    extern __shared__ uint32_t rm_smem[];  // ROW_MAJOR only: NW * rm_warp_words(U, SLOTS, ZREG) (none with TMEM and ZREG)
+    // ROW_MAJOR only: NW * rm_warp_words(U, SLOTS, ZREG) (TMEM: NW * ZS_WORDS, none with ZREG),
+    // then NW * TMA_BUF_WORDS when a.use_tma
+    extern __shared__ __align__(1024) uint32_t rm_smem[];
     __shared__ uint8_t* s_row0[LAYOUT == L_ROW_MAJOR ? BLOCK : 1];
     __shared__ uint32_t s_nvalid[LAYOUT == L_ROW_MAJOR ? BLOCK : 1];
     __shared__ uint64_t s_b0[LAYOUT == L_ROW_MAJOR ? NW : 1];
@@ -648,7 +722,13 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
                     const uint32_t t = tid_volatile();
                     const uint64_t col = (B - (k - k_lo)) * 4;
                     if constexpr (TMEM) {
-                        if (k_lo == 0 && k == 7 && ((a.row_bytes | col) & 7) == 0 && a.row_bytes < (1ull << 32))
+                        const uint64_t g_w0 = (*slot % a.units) * 32u;  // the warp's first group
+                        if (a.use_tma && k_lo == 0 && k == 7 && g_w0 + 32 <= a.tma_groups)
+                            rowmajor_store_tmem_tma(tm_addr(),
+                                                    rm_smem + NW * (U == 32 && ZREG ? 0 : ZS_WORDS) +
+                                                        (t >> 5) * TMA_BUF_WORDS,
+                                                    &a.tmap, g_w0, col);
+                        else if (k_lo == 0 && k == 7 && ((a.row_bytes | col) & 7) == 0 && a.row_bytes < (1ull << 32))
                             rowmajor_store_tmem_sectors(tm_addr(), s_row0 + (t & ~31u), s_nvalid + (t & ~31u),
                                                         a.row_bytes, col);
                         else
@@ -690,7 +770,11 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const KsArgs a)
         }
         next_item(a, slot);
     }
-    if constexpr (LAYOUT == L_ROW_MAJOR && TMEM) tmem_dealloc_cta(*reinterpret_cast<volatile uint32_t*>(&s_tmem));
+    if constexpr (LAYOUT == L_ROW_MAJOR && TMEM) {
+        if (a.use_tma && laneid_volatile() == 0) bulk_wait_all();  // smem boxes read, stores done
+        __syncwarp();
+        tmem_dealloc_cta(*reinterpret_cast<volatile uint32_t*>(&s_tmem));
+    }
 }
 
 }  // namespace bsk

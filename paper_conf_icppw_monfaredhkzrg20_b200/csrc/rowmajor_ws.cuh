@@ -65,7 +65,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity)
 }  // namespace ws
 
 template <class C, int U>
-__global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const KsArgs a)
+__global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __grid_constant__ KsArgs a)
 {
     static_assert(32 % U == 0, "U must divide 32");
     constexpr int KB = ks_block<C, U>();

@@ -142,6 +142,8 @@ def test_mickey_2_40_limit_boundary():
     ("grain", {"rm_tmem": 1, "ctas_per_sm": 2, "seg_clocks": 512}, 4096),
     ("mickey2", {"rm_ws": 0, "rm_tmem": 1}, 4416),
     ("mickey2", {"rm_ws": 0, "rm_tmem": 1, "seg_clocks": 96}, 1024),
+    ("grain", {"rm_tmem": 1, "rm_tma": 0}, 8192),        # 8 B global-store flush instead of TMA
+    ("mickey2", {"rm_ws": 0, "rm_tmem": 1}, 8192),        # TMA flush (1 KB rows) for warp 0, 8 B for warp 1
 ])
 def test_rm_tmem_staging_bit_exact(cipher, opts, bits):
     """ROW_MAJOR with the row segments staged in tensor memory (TMEM) instead
@@ -210,3 +212,19 @@ def test_device_input_rekey(cipher, n, misalign):
             return buf[3:3 + flat.numel()]
         g.rekey(dev(k), dev(ivs))
         assert np.array_equal(g.generate_host(bits, "row_major"), want), seed
+
+
+@pytest.mark.parametrize("cipher,bits,opts", [
+    ("grain", 4096, {}), ("grain", 2048, {"seg_clocks": 512}), ("mickey2", 2048, {}), ("grain", 4096, {"rm_tma": 0}),
+])
+def test_rm_tma_flush_many_warps(cipher, bits, opts):
+    """TMA tensor-store flushes (3-D view [q][group][byte] of the row-major
+    output) from several warp-units at once plus a ragged tail unit that
+    falls back to global stores: every row bit-exact."""
+    n = 32 * 32 * 4 + 17
+    keys, ivs = inputs.make_inputs(cipher, n)
+    want = _want(cipher, keys, ivs, bits)
+    g = _gen(cipher, keys, ivs)
+    for k, v in opts.items():
+        g.set_option(k, v)
+    assert np.array_equal(g.generate_host(bits, "row_major"), want)
