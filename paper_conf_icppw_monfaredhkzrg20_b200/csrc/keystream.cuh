@@ -523,38 +523,40 @@ __device__ __forceinline__ void tma_store_3d(const CUtensorMap* map, uint32_t sr
 }
 constexpr int TMA_BUF_WORDS = 4096;  // 16 KB per warp: two 8 KB boxes
 
-__device__ __forceinline__ void rowmajor_store_tmem_tma(uint32_t tm, uint32_t* buf, const CUtensorMap* map,
-                                                        uint64_t g_w0, uint64_t col)
+// One half of a TMA flush: TMEM lanes 16h..16h+15 (groups g_w0 + 16h ..
+// +15, two 8-group boxes).  The second half of a flush is deferred to the
+// start of the warp's next 32-clock block (before that block's transpose
+// overwrites slot 0), so the TMA engine has a block's worth of clocks to read
+// the first half's boxes out of the 16 KB buffer; waiting for those reads
+// right away cost 8.6% of Grain's ROW_MAJOR time (ncu: BSYNC after lane 0's
+// cp.async.bulk.wait_group.read).
+__device__ __forceinline__ void tma_flush_half(uint32_t tm, uint32_t* buf, const CUtensorMap* map, uint64_t g_w0,
+                                               uint64_t col, uint32_t h)
 {
-    tmem_wait_st();
     const uint32_t t = laneid_volatile();
     const uint32_t sb = smem_addr_u32(buf);
     const uint32_t off_t = (t >> 2) * 32 + (t & 3) * 8;
+    if (t == 0) bulk_wait_read_all();  // the previous boxes have left the buffer
+    __syncwarp();
 #pragma unroll 1
-    for (uint32_t h = 0; h < 2; ++h) {
-        // the previous TMA stores must have read the buffer
-        if (t == 0) bulk_wait_read_all();
-        __syncwarp();
-#pragma unroll 1
-        for (uint32_t q0 = 0; q0 < 32; q0 += 4) {
-            uint32_t v[16];
-            tmem_ld16x256b_x4(tm + ((16 * h) << 16) + q0 * 8, v);
+    for (uint32_t q0 = 0; q0 < 32; q0 += 4) {
+        uint32_t v[16];
+        tmem_ld16x256b_x4(tm + ((16 * h) << 16) + q0 * 8, v);
 #pragma unroll
-            for (int i = 0; i < 4; ++i) {
-                const uint32_t o = sb + (q0 + i) * 256 + off_t;
-                asm volatile("st.shared.v2.b32 [%0], {%1, %2};" ::"r"(o), "r"(v[4 * i]), "r"(v[4 * i + 1]) : "memory");
-                asm volatile("st.shared.v2.b32 [%0], {%1, %2};" ::"r"(o + 8192), "r"(v[4 * i + 2]), "r"(v[4 * i + 3])
-                             : "memory");
-            }
+        for (int i = 0; i < 4; ++i) {
+            const uint32_t o = sb + (q0 + i) * 256 + off_t;
+            asm volatile("st.shared.v2.b32 [%0], {%1, %2};" ::"r"(o), "r"(v[4 * i]), "r"(v[4 * i + 1]) : "memory");
+            asm volatile("st.shared.v2.b32 [%0], {%1, %2};" ::"r"(o + 8192), "r"(v[4 * i + 2]), "r"(v[4 * i + 3])
+                         : "memory");
         }
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic-proxy writes -> TMA reads
-        __syncwarp();
-        if (t == 0) {
-            const int g = int(g_w0 + 16 * h);
-            tma_store_3d(map, sb, int(col), g, 0);
-            tma_store_3d(map, sb + 8192, int(col), g + 8, 0);
-            asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-        }
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic-proxy writes -> TMA reads
+    __syncwarp();
+    if (t == 0) {
+        const int g = int(g_w0 + 16 * h);
+        tma_store_3d(map, sb, int(col), g, 0);
+        tma_store_3d(map, sb + 8192, int(col), g + 8, 0);
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
     }
 }
 
@@ -582,6 +584,9 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
     __shared__ uint32_t s_nvalid[LAYOUT == L_ROW_MAJOR ? BLOCK : 1];
     __shared__ uint64_t s_b0[LAYOUT == L_ROW_MAJOR ? NW : 1];
     __shared__ uint32_t s_nblk[LAYOUT == L_ROW_MAJOR ? NW : 1];
+    // TMA flush whose second half is pending (col + 1, 0 = none) and its first group
+    __shared__ uint64_t s_pend_col[LAYOUT == L_ROW_MAJOR && TMEM ? NW : 1];
+    __shared__ uint64_t s_pend_g[LAYOUT == L_ROW_MAJOR && TMEM ? NW : 1];
     __shared__ uint32_t s_item[NW];
     // Only `s_item` (smem) and the loop counters survive a clock loop; every
     // other per-item value is re-derived afterwards, so the 200 state words
@@ -594,9 +599,27 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
     if constexpr (LAYOUT == L_ROW_MAJOR && TMEM) {
         static_assert(BLOCK == 128, "TMEM staging maps warp w to lane quarter w");
         (void)tmem_alloc_cta(&s_tmem);
+        if (laneid_volatile() == 0) s_pend_col[threadIdx.x >> 5] = 0;
     }
     auto tm_addr = [&]() {
         return *reinterpret_cast<volatile uint32_t*>(&s_tmem) + ((threadIdx.x >> 5) << 21);
+    };
+    auto tma_buf = [&]() {
+        return rm_smem + NW * (U == 32 && ZREG ? 0 : ZS_WORDS) + (tid_volatile() >> 5) * TMA_BUF_WORDS;
+    };
+    // issue the deferred second half of the previous block's TMA flush
+    auto tma_pending = [&]() {
+        if constexpr (LAYOUT == L_ROW_MAJOR && TMEM) {
+            const uint32_t wq = tid_volatile() >> 5;
+            const uint64_t pc = *reinterpret_cast<volatile uint64_t*>(&s_pend_col[wq]);
+            if (pc) {
+                tma_flush_half(tm_addr(), tma_buf(), &a.tmap, *reinterpret_cast<volatile uint64_t*>(&s_pend_g[wq]),
+                               pc - 1, 1);
+                __syncwarp();
+                if (laneid_volatile() == 0) s_pend_col[wq] = 0;
+                __syncwarp();
+            }
+        }
     };
     if (a.persistent)
         next_item(a, slot);
@@ -694,6 +717,7 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
                     });
                     const uint64_t B = *reinterpret_cast<volatile uint64_t*>(&s_b0[tid_volatile() >> 5]) + blk;
                     const uint32_t k = uint32_t(B & (NSLOT - 1));
+                    tma_pending();
                     if constexpr (TMEM)
                         rowmajor_transpose_tmem<C::MSB_FIRST>(zr, tm_addr(), k);
                     else
@@ -710,6 +734,7 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
                     }
                     const uint64_t B = *reinterpret_cast<volatile uint64_t*>(&s_b0[tid_volatile() >> 5]) + blk;
                     const uint32_t k = uint32_t(B & (NSLOT - 1));
+                    tma_pending();
                     if constexpr (TMEM)
                         rowmajor_transpose_smem_tmem<C::MSB_FIRST>(zs_ptr(), tm_addr(), k);
                     else
@@ -723,12 +748,19 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
                     const uint64_t col = (B - (k - k_lo)) * 4;
                     if constexpr (TMEM) {
                         const uint64_t g_w0 = (*slot % a.units) * 32u;  // the warp's first group
-                        if (a.use_tma && k_lo == 0 && k == 7 && g_w0 + 32 <= a.tma_groups)
-                            rowmajor_store_tmem_tma(tm_addr(),
-                                                    rm_smem + NW * (U == 32 && ZREG ? 0 : ZS_WORDS) +
-                                                        (t >> 5) * TMA_BUF_WORDS,
-                                                    &a.tmap, g_w0, col);
-                        else if (k_lo == 0 && k == 7 && ((a.row_bytes | col) & 7) == 0 && a.row_bytes < (1ull << 32))
+                        if (a.use_tma && k_lo == 0 && k == 7 && g_w0 + 32 <= a.tma_groups) {
+                            tmem_wait_st();
+                            tma_flush_half(tm_addr(), tma_buf(), &a.tmap, g_w0, col, 0);
+                            if (blk + 1 < nblk) {  // defer the second half to the next block
+                                if (laneid_volatile() == 0) {
+                                    s_pend_col[t >> 5] = col + 1;
+                                    s_pend_g[t >> 5] = g_w0;
+                                }
+                                __syncwarp();
+                            } else {
+                                tma_flush_half(tm_addr(), tma_buf(), &a.tmap, g_w0, col, 1);
+                            }
+                        } else if (k_lo == 0 && k == 7 && ((a.row_bytes | col) & 7) == 0 && a.row_bytes < (1ull << 32))
                             rowmajor_store_tmem_sectors(tm_addr(), s_row0 + (t & ~31u), s_nvalid + (t & ~31u),
                                                         a.row_bytes, col);
                         else
