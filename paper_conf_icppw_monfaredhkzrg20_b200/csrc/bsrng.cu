@@ -455,7 +455,7 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
 // AES-CTR: persistent grid of one 4-warp CTA per SM; work items (time segment,
 // warp-unit) are independent, so segments need no flags (aes.cuh).
 template <int LAYOUT>
-int launch_aes(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
+int launch_aes(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st, uint64_t row_stride = 0, uint64_t t0_add = 0)
 {
     auto kern = &bsk::aes_ctr_kernel<LAYOUT>;
     bsk::KsArgs a{};
@@ -466,10 +466,10 @@ int launch_aes(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
     const uint64_t tail = h->n - (h->G - 1) * 32;
     a.tail_mask = tail >= 32 ? 0xFFFFFFFFu : ((1u << tail) - 1u);
     a.nclocks = bits;
-    a.t0 = h->bits_done;
+    a.t0 = h->bits_done + t0_add;
     a.g_base = h->first_instance / 32;
     a.out = out;
-    a.row_bytes = bits / 8;
+    a.row_bytes = row_stride ? row_stride : bits / 8;
     a.units = h->units;
     a.scratch = h->sched + 1 + h->units;
     a.persistent = 1;
@@ -510,7 +510,7 @@ int launch_aes(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
 }
 
 // AES ROW_MAJOR with >= 32 blocks per instance: block-lane kernel (aes.cuh).
-int launch_aes_rowmajor_lanes(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
+int launch_aes_rowmajor_lanes(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st, uint64_t row_stride = 0)
 {
     auto kern = &bsk::aes_ctr_rowmajor_lanes_kernel;
     bsk::KsArgs a{};
@@ -520,7 +520,7 @@ int launch_aes_rowmajor_lanes(bsrng_t* h, void* out, uint64_t bits, cudaStream_t
     a.nclocks = bits;
     a.t0 = h->bits_done;
     a.out = out;
-    a.row_bytes = bits / 8;
+    a.row_bytes = row_stride ? row_stride : bits / 8;
     a.units = h->G;  // one warp = 32 instances
     a.aux = h->raw + h->iv_off;
     a.persistent = 1;
@@ -740,10 +740,22 @@ int bsrng_generate(bsrng_t* h, void* out, uint64_t bits, bsrng_layout layout, vo
     case BSRNG_GRAIN_V1: rc = dispatch_layout<bsk::Grain>(h, out, bits, layout, st); break;
     case BSRNG_LFSR128: rc = dispatch_layout<bsk::Lfsr128>(h, out, bits, layout, st); break;
     case BSRNG_AES128_CTR:
-        rc = layout == BSRNG_ROW_MAJOR ? (bits >= 4096 && h->opt_rm_ws ? launch_aes_rowmajor_lanes(h, out, bits, st)
-                                                                       : launch_aes<bsk::L_ROW_MAJOR>(h, out, bits, st))
-             : layout == BSRNG_SLICED  ? launch_aes<bsk::L_SLICED>(h, out, bits, st)
-                                       : launch_aes<bsk::L_CHECKSUM>(h, out, bits, st);
+        if (layout == BSRNG_ROW_MAJOR && bits >= 4096 && h->opt_rm_ws) {
+            // whole 32-block encryptions per instance in the block-lane kernel
+            // (one instance per thread); a remainder of < 32 blocks would waste
+            // most of an encryption's lanes there (the paper-shape 35-block
+            // call ran at 0.44 of the roofline), so it goes to the
+            // instance-sliced kernel, writing the rows' last bytes
+            const uint64_t main_bits = bits / 4096 * 4096, rem = bits - main_bits;
+            rc = launch_aes_rowmajor_lanes(h, out, main_bits, st, bits / 8);
+            if (rc == BSRNG_OK && rem)
+                rc = launch_aes<bsk::L_ROW_MAJOR>(h, static_cast<uint8_t*>(out) + main_bits / 8, rem, st, bits / 8,
+                                                  main_bits);
+        } else {
+            rc = layout == BSRNG_ROW_MAJOR ? launch_aes<bsk::L_ROW_MAJOR>(h, out, bits, st)
+                 : layout == BSRNG_SLICED  ? launch_aes<bsk::L_SLICED>(h, out, bits, st)
+                                           : launch_aes<bsk::L_CHECKSUM>(h, out, bits, st);
+        }
         break;
     default: rc = fail(BSRNG_EUNSUPPORTED, "cipher not built");
     }

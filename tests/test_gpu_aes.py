@@ -112,3 +112,18 @@ def test_rowmajor_block_lanes(bits, seg):
     want = oracle.aes128_ctr_keystream_batch(bytes(key), ctrs, bits, first_block=3)
     assert np.array_equal(got, want)
     assert int(pre[0]) == checksum(to_sliced(oracle.aes128_ctr_keystream_batch(bytes(key), ctrs, 384)))
+
+
+@pytest.mark.parametrize("bits", [4480, 8192 + 128, 4096 + 31 * 128, 4096])
+def test_rowmajor_lanes_plus_remainder(bits):
+    """ROW_MAJOR calls of >= 32 blocks: whole 32-block encryptions in the
+    block-lane kernel, the < 32-block remainder in the instance-sliced kernel
+    writing the rows' last bytes (paper shape: 35 blocks = 4480 bits); two
+    consecutive calls continue the counters."""
+    n = 32 * 9 + 5
+    g, key, ctrs = _gen(n)
+    want = oracle.aes128_ctr_keystream_batch(bytes(key), ctrs, 2 * bits)
+    got1 = g.generate_host(bits, "row_major")
+    got2 = g.generate_host(bits, "row_major")
+    assert np.array_equal(got1, want[:, :bits // 8])
+    assert np.array_equal(got2, want[:, bits // 8:])
