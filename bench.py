@@ -255,13 +255,15 @@ def cpu_baseline(target_s=25.0, cipher="mickey2"):
 
 
 def run_context(local_rank):
-    """Live context numbers on this GPU: the measured LOP3 issue ceiling and
-    cuRAND on the same B200 (tools/microbench, built by __graft_entry__.build)."""
+    """Live context numbers on this GPU: the measured LOP3 issue ceiling,
+    cuRAND on the same B200 and the HBM write-only bandwidth (STG.128 /
+    STG.32 streams; tools/microbench, built by __graft_entry__.build)."""
     out = {}
     mb = os.path.join(ROOT, "tools", "microbench")
     env = dict(os.environ, CUDA_VISIBLE_DEVICES=os.environ.get("CUDA_VISIBLE_DEVICES", str(local_rank)))
-    for name, argv in (("alu_peak", ["200000"]), ("curand", ["4294967296"])):
-        exe = os.path.join(mb, "alu_peak" if name == "alu_peak" else "curand_bench")
+    exes = {"alu_peak": "alu_peak", "curand": "curand_bench", "write_peak": "write_peak"}
+    for name, argv in (("alu_peak", ["200000"]), ("curand", ["4294967296"]), ("write_peak", [])):
+        exe = os.path.join(mb, exes[name])
         if not os.path.exists(exe):
             out[name] = "not built"
             continue
@@ -272,6 +274,8 @@ def run_context(local_rank):
             out[name] = f"failed: {e}"
     if isinstance(out.get("alu_peak"), list) and out["alu_peak"]:
         out["alu_peak_tlop3_per_s"] = max(x["tlop3_per_s"] for x in out["alu_peak"] if x["variant"] == "lop3")
+    if isinstance(out.get("write_peak"), list) and out["write_peak"]:
+        out["hbm_write_peak_gbs"] = max(x["write_gbs"] for x in out["write_peak"])
     return out
 
 
