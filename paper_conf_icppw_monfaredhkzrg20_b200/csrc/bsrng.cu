@@ -110,6 +110,9 @@ struct bsrng {
     // TMEM-staged ROW_MAJOR: whole-sector flushes as TMA tensor stores (1) or
     // as 8 B global stores from the 16x256b read-back (0)
     int opt_rm_tma = 1;
+    // TMEM-staged ROW_MAJOR with one CTA per SM: double-buffered staging with
+    // the previous sector period flushed 4 rows per block (1) or not (0)
+    int opt_rm_dbl = 1;
     // init: slicing fused into the init kernel (MICKEY, Grain) / per-thread group
     // slicing into the state (AES, LFSR) (1), or the ballot slice kernels (0).
     int opt_init_fused = 1;
@@ -426,6 +429,10 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
         cudaError_t e = cudaMemsetAsync(h->sched, 0, (1 + h->units) * sizeof(uint32_t), st);
         if (e != cudaSuccess) return fail(BSRNG_ECUDA, "memset(sched): %s", cudaGetErrorString(e));
     }
+    // one CTA per SM and no time segments (no CTA ever waits on another, so a
+    // second CTA queued behind a 512-column allocation cannot deadlock): the
+    // lone clock-loop warps get double-buffered TMEM staging (KsArgs::tmem_dbl)
+    if (tmem && !a.use_tma && h->opt_rm_dbl && a.nseg == 1 && grid <= unsigned(h->num_sms)) a.tmem_dbl = 1;
     if (LAYOUT == bsk::L_CHECKSUM) {
         cudaError_t e = cudaMemsetAsync(out, 0, sizeof(uint64_t), st);
         if (e != cudaSuccess) return fail(BSRNG_ECUDA, "memset(out): %s", cudaGetErrorString(e));
@@ -864,6 +871,8 @@ int bsrng_set_option(bsrng_t* h, const char* key, int64_t value)
     } else if (!strcmp(key, "rm_zreg")) {
         if (value != 0 && value != 1) return fail(BSRNG_EINVAL, "rm_zreg must be 0 or 1");
         h->opt_rm_zreg = int(value);
+    } else if (!strcmp(key, "rm_dbl")) {
+        h->opt_rm_dbl = int(value);
     } else if (!strcmp(key, "rm_tma")) {
         h->opt_rm_tma = int(value);
     } else if (!strcmp(key, "rm_tmem")) {

@@ -113,6 +113,11 @@ struct KsArgs {
     // ROW_MAJOR + TMEM: whole-sector flushes of warps whose 32 groups are all
     // real (g < tma_groups) go out as TMA tensor stores (rowmajor_store_tmem_tma)
     int use_tma;
+    // ROW_MAJOR + TMEM with one CTA per SM (grid <= SMs, no time segments):
+    // 512 columns = two staging buffers; a completed sector period is
+    // flushed 4 rows per block during the next period (lone clock-loop warps
+    // cannot otherwise hide the flush)
+    int tmem_dbl;
     uint64_t tma_groups;
     CUtensorMap tmap;  // 3-D view of `out`: [q 32][group][byte], see bsrng.cu
 };
@@ -276,13 +281,17 @@ __device__ __forceinline__ void rowmajor_store(const uint32_t* os, uint8_t* row0
 // ---------------------------------------------------------------------------
 constexpr uint32_t TMEM_COLS = 256;
 
-__device__ __forceinline__ uint32_t tmem_alloc_cta(uint32_t* s_base)
+// dbl: 512 columns (two staging buffers; one CTA per SM, see KsArgs::tmem_dbl)
+__device__ __forceinline__ uint32_t tmem_alloc_cta(uint32_t* s_base, bool dbl = false)
 {
     if ((threadIdx.x >> 5) == 0) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
-                         static_cast<uint32_t>(__cvta_generic_to_shared(s_base))),
-                     "n"(TMEM_COLS)
-                     : "memory");
+        const uint32_t sb = static_cast<uint32_t>(__cvta_generic_to_shared(s_base));
+        if (dbl)
+            asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(sb), "n"(2 * TMEM_COLS)
+                         : "memory");
+        else
+            asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(sb), "n"(TMEM_COLS)
+                         : "memory");
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
     }
     asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
@@ -291,13 +300,19 @@ __device__ __forceinline__ uint32_t tmem_alloc_cta(uint32_t* s_base)
     return *reinterpret_cast<volatile uint32_t*>(s_base);
 }
 
-__device__ __forceinline__ void tmem_dealloc_cta(uint32_t base)
+__device__ __forceinline__ void tmem_dealloc_cta(uint32_t base, bool dbl = false)
 {
     asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
     __syncthreads();
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-    if ((threadIdx.x >> 5) == 0)
-        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(base), "n"(TMEM_COLS) : "memory");
+    if ((threadIdx.x >> 5) == 0) {
+        if (dbl)
+            asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(base), "n"(2 * TMEM_COLS)
+                         : "memory");
+        else
+            asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(base), "n"(TMEM_COLS)
+                         : "memory");
+    }
 }
 
 // column taddr + OFF of this thread's lane <- v (one uniform base register,
@@ -508,6 +523,34 @@ __device__ __forceinline__ void rowmajor_store_tmem_sectors(uint32_t tm, uint8_t
 // sector, laid out in smem as [q][group][32 B] so a 16x256b fragment (8
 // groups x 32 B for one q) is 256 contiguous bytes: conflict-free 8 B stores.
 // ---------------------------------------------------------------------------
+// Rows q in [q_lo, q_hi) (multiples of 4) of a whole-sector period, every
+// row real and 8 B aligned (tmem_dbl's progressive flush): 16x256b read-back,
+// unpredicated 8 B stores.
+__device__ __forceinline__ void rowmajor_store_tmem_rows(uint32_t tm, uint8_t* const* row0s, uint64_t row_bytes,
+                                                         uint64_t col, uint32_t q_lo, uint32_t q_hi)
+{
+    tmem_wait_st();
+    const uint32_t t = laneid_volatile();
+#pragma unroll 1
+    for (uint32_t h = 0; h < 2; ++h) {
+        const uint32_t la = 16 * h + (t >> 2), lb = la + 8;
+        uint8_t* pa = row0s[la] + col + 8 * (t & 3) + q_lo * row_bytes;
+        uint8_t* pb = row0s[lb] + col + 8 * (t & 3) + q_lo * row_bytes;
+#pragma unroll 1
+        for (uint32_t q0 = q_lo; q0 < q_hi; q0 += 4) {
+            uint32_t v[16];
+            tmem_ld16x256b_x4(tm + ((16 * h) << 16) + q0 * 8, v);
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+                __stcs(reinterpret_cast<uint2*>(pa), make_uint2(v[4 * i], v[4 * i + 1]));
+                __stcs(reinterpret_cast<uint2*>(pb), make_uint2(v[4 * i + 2], v[4 * i + 3]));
+                pa += row_bytes;
+                pb += row_bytes;
+            }
+        }
+    }
+}
+
 __device__ __forceinline__ uint32_t smem_addr_u32(const void* p)
 {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -587,6 +630,8 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
     // TMA flush whose second half is pending (col + 1, 0 = none) and its first group
     __shared__ uint64_t s_pend_col[LAYOUT == L_ROW_MAJOR && TMEM ? NW : 1];
     __shared__ uint64_t s_pend_g[LAYOUT == L_ROW_MAJOR && TMEM ? NW : 1];
+    // tmem_dbl: the previous sector period still being flushed (col + 1, 0 = none)
+    __shared__ uint64_t s_pdbl_col[LAYOUT == L_ROW_MAJOR && TMEM ? NW : 1];
     __shared__ uint32_t s_item[NW];
     // Only `s_item` (smem) and the loop counters survive a clock loop; every
     // other per-item value is re-derived afterwards, so the 200 state words
@@ -598,9 +643,11 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
     __shared__ uint32_t s_tmem;
     if constexpr (LAYOUT == L_ROW_MAJOR && TMEM) {
         static_assert(BLOCK == 128, "TMEM staging maps warp w to lane quarter w");
-        (void)tmem_alloc_cta(&s_tmem);
-        if (laneid_volatile() == 0) s_pend_col[threadIdx.x >> 5] = 0;
+        (void)tmem_alloc_cta(&s_tmem, a.tmem_dbl != 0);
+        if (laneid_volatile() == 0) s_pend_col[threadIdx.x >> 5] = s_pdbl_col[threadIdx.x >> 5] = 0;
     }
+    // tmem_dbl: sector period B >> 3 stages into buffer (B >> 3) & 1
+    auto dbl_off = [&](uint64_t B) -> uint32_t { return a.tmem_dbl ? uint32_t((B >> 3) & 1) * TMEM_COLS : 0u; };
     auto tm_addr = [&]() {
         return *reinterpret_cast<volatile uint32_t*>(&s_tmem) + ((threadIdx.x >> 5) << 21);
     };
@@ -719,7 +766,7 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
                     const uint32_t k = uint32_t(B & (NSLOT - 1));
                     tma_pending();
                     if constexpr (TMEM)
-                        rowmajor_transpose_tmem<C::MSB_FIRST>(zr, tm_addr(), k);
+                        rowmajor_transpose_tmem<C::MSB_FIRST>(zr, tm_addr() + dbl_off(B), k);
                     else
                         rowmajor_transpose_regs<C::MSB_FIRST, SLOTS>(zr, os_ptr(), k);
                 } else {
@@ -736,19 +783,44 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
                     const uint32_t k = uint32_t(B & (NSLOT - 1));
                     tma_pending();
                     if constexpr (TMEM)
-                        rowmajor_transpose_smem_tmem<C::MSB_FIRST>(zs_ptr(), tm_addr(), k);
+                        rowmajor_transpose_smem_tmem<C::MSB_FIRST>(zs_ptr(), tm_addr() + dbl_off(B), k);
                     else
                         rowmajor_transpose<C::MSB_FIRST, SLOTS>(zs_ptr(), os_ptr(), k);
                 }
                 const uint64_t B = *reinterpret_cast<volatile uint64_t*>(&s_b0[tid_volatile() >> 5]) + blk;
                 const uint32_t k = uint32_t(B & (NSLOT - 1));
+                if constexpr (TMEM) {
+                    // tmem_dbl: 4 rows of the previous period per block (the rest
+                    // at the item's last block), from the other buffer
+                    if (a.tmem_dbl) {
+                        const uint32_t wq = tid_volatile() >> 5;
+                        const uint64_t pc = *reinterpret_cast<volatile uint64_t*>(&s_pdbl_col[wq]);
+                        if (pc) {
+                            const uint32_t q_hi = blk + 1 == nblk ? 32u : 4 * k + 4;
+                            rowmajor_store_tmem_rows(tm_addr() + (dbl_off(B) ^ TMEM_COLS), s_row0 + wq * 32,
+                                                     a.row_bytes, pc - 1, 4 * k, q_hi);
+                            if (q_hi == 32) {
+                                __syncwarp();
+                                if (laneid_volatile() == 0) s_pdbl_col[wq] = 0;
+                                __syncwarp();
+                            }
+                        }
+                    }
+                }
                 if (k == NSLOT - 1 || blk + 1 == nblk) {
                     const uint32_t k_lo = k - (blk < k ? blk : k);
                     const uint32_t t = tid_volatile();
                     const uint64_t col = (B - (k - k_lo)) * 4;
                     if constexpr (TMEM) {
                         const uint64_t g_w0 = (*slot % a.units) * 32u;  // the warp's first group
-                        if (a.use_tma && k_lo == 0 && k == 7 && g_w0 + 32 <= a.tma_groups) {
+                        const bool full_real = __all_sync(0xFFFFFFFFu, s_nvalid[t] == 32);
+                        if (a.tmem_dbl && k_lo == 0 && k == 7 && blk + 1 < nblk && full_real &&
+                            ((a.row_bytes | col) & 7) == 0) {
+                            // flushed during the next period (other buffer)
+                            __syncwarp();
+                            if (laneid_volatile() == 0) s_pdbl_col[t >> 5] = col + 1;
+                            __syncwarp();
+                        } else if (a.use_tma && k_lo == 0 && k == 7 && g_w0 + 32 <= a.tma_groups) {
                             tmem_wait_st();
                             tma_flush_half(tm_addr(), tma_buf(), &a.tmap, g_w0, col, 0);
                             if (blk + 1 < nblk) {  // defer the second half to the next block
@@ -761,10 +833,11 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
                                 tma_flush_half(tm_addr(), tma_buf(), &a.tmap, g_w0, col, 1);
                             }
                         } else if (k_lo == 0 && k == 7 && ((a.row_bytes | col) & 7) == 0 && a.row_bytes < (1ull << 32))
-                            rowmajor_store_tmem_sectors(tm_addr(), s_row0 + (t & ~31u), s_nvalid + (t & ~31u),
-                                                        a.row_bytes, col);
+                            rowmajor_store_tmem_sectors(tm_addr() + dbl_off(B), s_row0 + (t & ~31u),
+                                                        s_nvalid + (t & ~31u), a.row_bytes, col);
                         else
-                            rowmajor_store_tmem(tm_addr(), s_row0[t], a.row_bytes, s_nvalid[t], k_lo, k, col);
+                            rowmajor_store_tmem(tm_addr() + dbl_off(B), s_row0[t], a.row_bytes, s_nvalid[t], k_lo, k,
+                                                col);
                     }
                     else
                         rowmajor_store<SLOTS>(os_ptr(), s_row0[t], a.row_bytes, s_nvalid[t], k_lo, k, col);
@@ -805,7 +878,7 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
     if constexpr (LAYOUT == L_ROW_MAJOR && TMEM) {
         if (a.use_tma && laneid_volatile() == 0) bulk_wait_all();  // smem boxes read, stores done
         __syncwarp();
-        tmem_dealloc_cta(*reinterpret_cast<volatile uint32_t*>(&s_tmem));
+        tmem_dealloc_cta(*reinterpret_cast<volatile uint32_t*>(&s_tmem), a.tmem_dbl != 0);
     }
 }
 

@@ -144,6 +144,9 @@ def test_mickey_2_40_limit_boundary():
     ("mickey2", {"rm_ws": 0, "rm_tmem": 1, "seg_clocks": 96}, 1024),
     ("grain", {"rm_tmem": 1, "rm_tma": 0}, 8192),        # 8 B global-store flush instead of TMA
     ("mickey2", {"rm_ws": 0, "rm_tmem": 1}, 8192),        # TMA flush (1 KB rows) for warp 0, 8 B for warp 1
+    ("grain", {"rm_tmem": 1, "rm_tma": 0}, 4416 + 256),  # double-buffered staging, progressive flush
+    ("mickey2", {"rm_ws": 0, "rm_tmem": 1, "rm_tma": 0}, 2048 + 96),  # ... item ends mid-period
+    ("grain", {"rm_tmem": 1, "rm_dbl": 0}, 4416),          # single buffer
 ])
 def test_rm_tmem_staging_bit_exact(cipher, opts, bits):
     """ROW_MAJOR with the row segments staged in tensor memory (TMEM) instead
