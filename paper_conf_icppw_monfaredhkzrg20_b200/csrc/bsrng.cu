@@ -291,15 +291,15 @@ int encode_rowmajor_tmap(CUtensorMap* map, void* out, uint64_t row_bytes, uint64
 }
 
 // Kernel instance for the handle's unroll option and ROW_MAJOR staging slots.
-template <class C, int LAYOUT, int SLOTS, bool ZREG = true, bool TMEM = false>
+template <class C, int LAYOUT, int SLOTS, bool ZREG = true, bool TMEM = false, bool DBL = false>
 auto pick_keystream_kernel(const bsrng_t* h, int* U)
 {
-    auto kern = &bsk::keystream_kernel<C, LAYOUT, C::U_DEFAULT, KS_BLOCK, SLOTS, ZREG, TMEM>;
+    auto kern = &bsk::keystream_kernel<C, LAYOUT, C::U_DEFAULT, KS_BLOCK, SLOTS, ZREG, TMEM, DBL>;
     *U = C::U_DEFAULT;
     if (h->opt_unroll == C::U_ALT0)
-        kern = &bsk::keystream_kernel<C, LAYOUT, C::U_ALT0, KS_BLOCK, SLOTS, true, TMEM>, *U = C::U_ALT0;
+        kern = &bsk::keystream_kernel<C, LAYOUT, C::U_ALT0, KS_BLOCK, SLOTS, true, TMEM, DBL>, *U = C::U_ALT0;
     if (h->opt_unroll == C::U_ALT1)
-        kern = &bsk::keystream_kernel<C, LAYOUT, C::U_ALT1, KS_BLOCK, SLOTS, true, TMEM>, *U = C::U_ALT1;
+        kern = &bsk::keystream_kernel<C, LAYOUT, C::U_ALT1, KS_BLOCK, SLOTS, true, TMEM, DBL>, *U = C::U_ALT1;
     return kern;
 }
 
@@ -432,7 +432,16 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
     // one CTA per SM and no time segments (no CTA ever waits on another, so a
     // second CTA queued behind a 512-column allocation cannot deadlock): the
     // lone clock-loop warps get double-buffered TMEM staging (KsArgs::tmem_dbl)
-    if (tmem && !a.use_tma && h->opt_rm_dbl && a.nseg == 1 && grid <= unsigned(h->num_sms)) a.tmem_dbl = 1;
+    if (LAYOUT == bsk::L_ROW_MAJOR && tmem && !a.use_tma && h->opt_rm_dbl && a.nseg == 1 &&
+        grid <= unsigned(h->num_sms)) {
+        a.tmem_dbl = 1;
+        kern = zreg ? pick_keystream_kernel<C, LAYOUT, 8, true, true, true>(h, &U)
+                    : pick_keystream_kernel<C, LAYOUT, 8, false, true, true>(h, &U);
+        if (smem > 48 * 1024) {
+            cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+            if (e != cudaSuccess) return fail(BSRNG_ECUDA, "smem attribute: %s", cudaGetErrorString(e));
+        }
+    }
     if (LAYOUT == bsk::L_CHECKSUM) {
         cudaError_t e = cudaMemsetAsync(out, 0, sizeof(uint64_t), st);
         if (e != cudaSuccess) return fail(BSRNG_ECUDA, "memset(out): %s", cudaGetErrorString(e));
