@@ -173,8 +173,15 @@ int64_t bsrng_copy_state(const bsrng_t* h, uint32_t* host_out, uint64_t words);
  *                  shared memory (0)
  *   "rm_tmem"    : ROW_MAJOR plain kernel: stage the row segments in tensor
  *                  memory (TMEM, 256 columns per CTA, two CTAs per SM) (1)
- *                  or in shared memory (0); -1 = cipher default (Grain 1,
- *                  MICKEY / LFSR 0)
+ *                  or in shared memory (0); -1 = cipher default (MICKEY /
+ *                  Grain 1, LFSR 0)
+ *   "rm_tma"     : TMEM staging: whole-sector flushes of warps whose rows are
+ *                  all real as TMA tensor stores when the row stride is a
+ *                  multiple of 16 B (1, default) or as 8 B stores (0)
+ *   "rm_dbl"     : TMEM staging with one CTA per SM and one work item per
+ *                  warp-unit: double-buffered staging (512 columns), the
+ *                  previous sector period flushed 4 rows per block (1,
+ *                  default) or a single buffer (0)
  *   "init_fused" : MICKEY / Grain create/rekey: slicing fused into the
  *                  initialisation kernel (1, default) or the separate
  *                  slice_bits + preclock kernels (0)
