@@ -13,7 +13,7 @@ Sweeps, for bitsliced MICKEY 2.0 (and a slice for Grain v1 / AES-128-CTR):
 Every point is CUDA-event timed on a warmed stream (best of `--reps`), with the
 algorithmic LOP3 rate against the ALU roofline at the SM clock sampled by
 nvidia-smi during the run.  cuRAND on the same byte count is timed by
-tools/microbench/curand_bench (context, printed by tools/gpu_sweep_c5.sh).
+tools/microbench/curand_bench (context, run by tools/gpu_c5.sh).
 
 Output: one JSON object per line (stdout).
 """
