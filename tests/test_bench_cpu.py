@@ -130,3 +130,21 @@ def test_mickey2_deferred_reduction_equals_galois_clocking():
                     low ^= Q[m]
             assert P >> (100 + k) == 0
             assert low == g and seen_l == seen_g
+
+
+def test_reference_arm_under_torchrun_world2():
+    """The driver launches the reference arm like ours for N > 1: rank 0 alone
+    runs the oracle and prints the one JSON line, the other rank exits 0."""
+    import socket
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+                        "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.join(ROOT, "bench.py"),
+                        "--impl", "reference", "--gpus", "2", "--steps", "1", "--warmup", "0"],
+                       capture_output=True, text=True, timeout=600, cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, r.stdout
+    line = json.loads(lines[0])
+    assert line["impl"] == "reference" and line["value"] > 0 and line["n_gpus"] == 2
