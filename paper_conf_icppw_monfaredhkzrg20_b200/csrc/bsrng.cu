@@ -196,7 +196,8 @@ int run_init(bsrng_t* h, cudaStream_t st, const uint8_t* raw_k, const uint8_t* r
                 if (e != cudaSuccess) return fail(BSRNG_ECUDA, "smem attribute: %s", cudaGetErrorString(e));
                 gattr = true;
             }
-            bsk::grain_init_kernel<<<blocks, 128, bsk::GI_SMEM_BYTES, st>>>(raw_k, raw_iv, tail_k, tail_iv, g_split,
+            bsk::grain_init_kernel<<<unsigned((h->Gp + GI_BLOCK - 1) / GI_BLOCK), GI_BLOCK, bsk::GI_SMEM_BYTES, st>>>(
+                raw_k, raw_iv, tail_k, tail_iv, g_split,
                                                                            h->state, h->Gp);
             return check_launch("grain_init");
         }

@@ -188,9 +188,12 @@ constexpr int GI_KSTRIDE = 336, GI_VSTRIDE = 272;
 #ifndef GI_UNROLL
 #define GI_UNROLL 40
 #endif
-constexpr size_t GI_SMEM_BYTES = size_t(128) * (GI_KSTRIDE + GI_VSTRIDE);  // 76 KB per 4-warp CTA
+#ifndef GI_BLOCK
+#define GI_BLOCK 128
+#endif
+constexpr size_t GI_SMEM_BYTES = size_t(GI_BLOCK) * (GI_KSTRIDE + GI_VSTRIDE);  // 19 KB per warp
 
-__global__ void __launch_bounds__(128) grain_init_kernel(const uint8_t* __restrict__ raw_k,
+__global__ void __launch_bounds__(GI_BLOCK) grain_init_kernel(const uint8_t* __restrict__ raw_k,
                                                          const uint8_t* __restrict__ raw_iv,
                                                          const uint8_t* __restrict__ tail_k,
                                                          const uint8_t* __restrict__ tail_iv, uint64_t g_split,
