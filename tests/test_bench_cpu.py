@@ -148,3 +148,18 @@ def test_reference_arm_under_torchrun_world2():
     assert len(lines) == 1, r.stdout
     line = json.loads(lines[0])
     assert line["impl"] == "reference" and line["value"] > 0 and line["n_gpus"] == 2
+
+
+def test_roofline_traffic_from_committed_captures():
+    """roofline.traffic comes from the committed ncu capture of the same
+    cipher and mode (profiles/keystream_traffic.json); materialise writes
+    scale with the bits per launch."""
+    for cipher, mode, bits in [("mickey2", "consume", 1 << 20), ("mickey2", "materialise", 1 << 15),
+                               ("grain", "consume", 1 << 20), ("grain", "materialise", 1 << 15),
+                               ("aes128ctr", "materialise", 1 << 15)]:
+        t, note = bench.traffic_for(cipher, mode, 1 << 22, bits)
+        assert t is not None and t > 0 and note, (cipher, mode)
+        if mode == "materialise":
+            alg = (1 << 22) * bits / 8
+            assert 0.95 * alg < t < 1.2 * alg, (cipher, t / alg)   # ~1.0x the keystream bytes
+    assert bench.traffic_for("mickey2", "consume", 1 << 19, 1 << 20) == (None, None)  # other n: no capture
