@@ -56,7 +56,9 @@ def lop3_per_bit(cipher, mode, unroll=None):
     if cipher == "grain":
         return 38.0 if mode == "consume" else 37.0
     if cipher == "lfsr128":
-        return 3.0 if mode == "consume" else 2.0
+        # feedback XOR4 = 2 LOP3; consume folds two clocks' output words into
+        # the accumulator with one XOR3 (0.5 per clock; 128-clock loop body)
+        return 2.5 if mode == "consume" else 2.0
     return (17280.0 + (64.0 if mode == "consume" else 0.0)) / 128.0
 CIPHER_NAME = {"mickey2": "MICKEY 2.0", "grain": "Grain v1", "aes128ctr": "AES-128-CTR",
                "lfsr128": "bitsliced LFSR-128 (Eq. 2)"}

@@ -52,6 +52,15 @@ __host__ __device__ constexpr int ks_block()
     else
         return 1;
 }
+// Consume-mode clocks per iteration for ciphers whose register rotation
+// closes after a short period (Lfsr128: 128 clocks, 3 LOP3 per clock): a body
+// of the full period needs no rotation moves, which at U = 32 outnumber the
+// logic (4 moves per clock).  0 = use U.
+template <class C, class = void>
+struct ks_u_big : std::integral_constant<int, 0> {};
+template <class C>
+struct ks_u_big<C, std::void_t<decltype(C::U_CONSUME)>> : std::integral_constant<int, C::U_CONSUME> {};
+
 template <int J, int K, class C>
 __device__ __forceinline__ uint32_t ks_z(const C& c)
 {
@@ -711,8 +720,21 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
         if (LAYOUT == L_CHECKSUM && seg > 0) acc = __ldcg(a.state + uint64_t(C::NSTATE) * a.Gp + g);
 
         if (LAYOUT == L_CHECKSUM) {
+            uint32_t nrem = nclk;
+            if constexpr (ks_u_big<C>::value > 0) {
+                constexpr int UB = ks_u_big<C>::value;
+                static_assert(KB == 1, "long consume bodies only for unphased ciphers");
 #pragma unroll 1
-            for (uint32_t it = nclk / U; it != 0; --it) {
+                for (uint32_t it = nclk / UB; it != 0; --it) {
+                    static_for<UB>([&](auto) {
+                        acc = ks_z_acc<0, 1>(c, acc);
+                        ks_clock<0, 1>(c);
+                    });
+                }
+                nrem = nclk % UB;
+            }
+#pragma unroll 1
+            for (uint32_t it = nrem / U; it != 0; --it) {
                 static_for<U>([&](auto u) {
                     constexpr int J = decltype(u)::value % KB;
                     acc = ks_z_acc<J, KB>(c, acc);

@@ -22,6 +22,8 @@ struct Lfsr128 {
     static constexpr bool MSB_FIRST = true;
     static constexpr int U_DEFAULT = 32, U_ALT0 = 8, U_ALT1 = 16;
     static constexpr bool RM_TMEM = false, RM_SEGMENTED = true;
+    // consume: one 128-clock body (the rotation period), no moves (keystream.cuh)
+    static constexpr int U_CONSUME = 128;
     uint32_t s[128];
 
     __device__ __forceinline__ void load(const uint32_t* st, uint64_t Gp, uint64_t g)
