@@ -724,14 +724,17 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
             if constexpr (ks_u_big<C>::value > 0) {
                 constexpr int UB = ks_u_big<C>::value;
                 static_assert(KB == 1, "long consume bodies only for unphased ciphers");
+                // the remainder must be whole U-clock iterations: split at a
+                // multiple of lcm(UB, 32)
+                constexpr uint32_t L = UB % 32 == 0 ? UB : (UB % 16 == 0 ? 2 * UB : 4 * UB);
+                nrem = nclk % L;
 #pragma unroll 1
-                for (uint32_t it = nclk / UB; it != 0; --it) {
+                for (uint32_t it = (nclk - nrem) / UB; it != 0; --it) {
                     static_for<UB>([&](auto) {
                         acc = ks_z_acc<0, 1>(c, acc);
                         ks_clock<0, 1>(c);
                     });
                 }
-                nrem = nclk % UB;
             }
 #pragma unroll 1
             for (uint32_t it = nrem / U; it != 0; --it) {
