@@ -60,6 +60,12 @@ template <class C, class = void>
 struct ks_u_big : std::integral_constant<int, 0> {};
 template <class C>
 struct ks_u_big<C, std::void_t<decltype(C::U_CONSUME)>> : std::integral_constant<int, C::U_CONSUME> {};
+// A cipher whose consume body is a whole period may supply consume_period(acc)
+// (Lfsr128: outputs folded from the entry state, clocks in place).
+template <class C, class = void>
+struct ks_period : std::false_type {};
+template <class C>
+struct ks_period<C, std::void_t<decltype(C::CONSUME_PERIOD)>> : std::integral_constant<bool, C::CONSUME_PERIOD> {};
 
 template <int J, int K, class C>
 __device__ __forceinline__ uint32_t ks_z(const C& c)
@@ -730,10 +736,14 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
                 nrem = nclk % L;
 #pragma unroll 1
                 for (uint32_t it = (nclk - nrem) / UB; it != 0; --it) {
-                    static_for<UB>([&](auto) {
-                        acc = ks_z_acc<0, 1>(c, acc);
-                        ks_clock<0, 1>(c);
-                    });
+                    if constexpr (ks_period<C>::value) {
+                        c.consume_period(acc);
+                    } else {
+                        static_for<UB>([&](auto) {
+                            acc = ks_z_acc<0, 1>(c, acc);
+                            ks_clock<0, 1>(c);
+                        });
+                    }
                 }
             }
 #pragma unroll 1

@@ -24,6 +24,7 @@ struct Lfsr128 {
     static constexpr bool RM_TMEM = false, RM_SEGMENTED = true;
     // consume: one 128-clock body (the rotation period), no moves (keystream.cuh)
     static constexpr int U_CONSUME = 128;
+    static constexpr bool CONSUME_PERIOD = true;
     uint32_t s[128];
 
     __device__ __forceinline__ void load(const uint32_t* st, uint64_t Gp, uint64_t g)
@@ -40,6 +41,32 @@ struct Lfsr128 {
     }
     __device__ __forceinline__ uint32_t z() const { return s[0]; }
     __device__ __forceinline__ uint32_t z_acc(uint32_t acc) const { return acc ^ s[0]; }
+    // One consume period: 128 clocks with their output words XORed into acc.
+    // The outputs of clocks t = 0..127 are z_t = s_t, i.e. exactly the 128
+    // state words at entry, so they are folded first (43 XOR3 in a 3-ary
+    // tree) and the 128 clocks then run in place: register t takes s_{t+128}
+    // = s_t ^ s_{t+2} ^ s_{t+27} ^ s_{t+29}, whose operands sit in registers
+    // (t+k) mod 128 (already overwritten iff t+k >= 128, which is then the
+    // needed s_{t+k}).  Same 2.5 ops per clock as the per-clock form, but no
+    // register outlives its clock, so no moves.
+    __device__ __forceinline__ void consume_period(uint32_t& acc)
+    {
+        uint32_t r[43];
+#pragma unroll
+        for (int i = 0; i < 42; ++i) r[i] = lop3<0x96u>(s[3 * i], s[3 * i + 1], s[3 * i + 2]);
+        r[42] = lop3<0x96u>(s[126], s[127], acc);
+        uint32_t q[15];
+#pragma unroll
+        for (int i = 0; i < 14; ++i) q[i] = lop3<0x96u>(r[3 * i], r[3 * i + 1], r[3 * i + 2]);
+        q[14] = r[42];
+        uint32_t p[5];
+#pragma unroll
+        for (int i = 0; i < 5; ++i) p[i] = lop3<0x96u>(q[3 * i], q[3 * i + 1], q[3 * i + 2]);
+        acc = lop3<0x96u>(lop3<0x96u>(p[0], p[1], p[2]), p[3], p[4]);
+#pragma unroll
+        for (int t = 0; t < 128; ++t)
+            s[t] = lop3<0x96u>(lop3<0x96u>(s[(t + 29) & 127], s[(t + 27) & 127], s[(t + 2) & 127]), s[t], 0u);
+    }
     __device__ __forceinline__ void clock()
     {
         const uint32_t fb = lop3<0x96u>(lop3<0x96u>(s[29], s[27], s[2]), s[0], 0u);
