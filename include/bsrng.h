@@ -63,17 +63,26 @@ typedef enum {
 
 enum {
     BSRNG_OK = 0,
-    BSRNG_EINVAL = -1,      /* bad argument (NULL, n == 0, bits % 32, layout, alignment) */
-    BSRNG_ENOMEM = -2,      /* device allocation failed                                   */
+    BSRNG_EINVAL = -1,      /* bad argument (NULL, n == 0, bits % 32, layout, alignment,
+                               iv_bits, a stream of another device)                      */
+    BSRNG_ENOMEM = -2,      /* device / pinned-host allocation failed, or all 11 AES
+                               round-key slots are taken (one per live AES handle)       */
     BSRNG_ECUDA = -3,       /* CUDA launch/runtime error (message in last_error)          */
-    BSRNG_ERANGE = -4,      /* would exceed 2^40 keystream bits per key/IV */
+    BSRNG_ERANGE = -4,      /* cumulative keystream bits per key/IV would exceed the
+                               cipher's limit: MICKEY 2.0 2^40 (the spec's limit,
+                               PAPER.md:254-256, reading R10); Grain v1, AES-128-CTR
+                               and the LFSR 2^62 (the 64-bit bit counter)               */
     BSRNG_EUNSUPPORTED = -5 /* cipher/layout combination not built                        */
 };
 
 /* flags for bsrng_create_ex / bsrng_rekey */
 enum {
-    BSRNG_INPUT_HOST = 0,   /* keys/ivs are host pointers (copied H2D, stream-ordered) */
-    BSRNG_INPUT_DEVICE = 1  /* keys/ivs are device pointers (no copy)                  */
+    BSRNG_INPUT_HOST = 0,   /* keys/ivs are host pointers: copied into a handle-owned
+                               pinned buffer during the call, then H2D stream-ordered;
+                               the caller may reuse its buffers as soon as it returns  */
+    BSRNG_INPUT_DEVICE = 1  /* keys/ivs are device pointers on the handle's device,
+                               read by kernels on `stream`: they must stay unchanged
+                               until the stream has passed the call                   */
 };
 
 typedef struct bsrng bsrng_t;
@@ -94,13 +103,18 @@ bsrng_t* bsrng_create(bsrng_cipher cipher, const uint8_t* keys, const uint8_t* i
 
 /*
  * bsrng_create_ex -- as bsrng_create, plus:
- *   iv_bits          : MICKEY IV length in bits, 0..80, multiple of 8 (IV row
- *                      stride is still 10 B); Grain must be 64; AES 128; LFSR 0.
+ *   iv_bits          : MICKEY IV length in bits, any value in 0..80 (the spec's
+ *                      range; IV bit i = bit 7 - i%8 of byte
+ *                      i/8; the IV row stride is still 10 B); Grain must be 64;
+ *                      AES 128; LFSR 0.
  *   first_instance_id: global id of instance 0 (must be a multiple of 32); used
  *                      only to make CHECKSUM shard-invariant.
  *   flags            : BSRNG_INPUT_HOST or BSRNG_INPUT_DEVICE.
- *   stream           : work is enqueued on `stream`; the call synchronises it
+ *   stream           : work is enqueued on `stream` (which must belong to the
+ *                      current device, else EINVAL); the call synchronises it
  *                      before returning.
+ * AES-128-CTR handles each take one of 11 constant-memory round-key slots
+ * (released by bsrng_destroy); a 12th live AES handle fails with ENOMEM.
  */
 bsrng_t* bsrng_create_ex(bsrng_cipher cipher, const uint8_t* keys, const uint8_t* ivs,
                          uint32_t iv_bits, uint64_t n, uint64_t first_instance_id,
@@ -109,8 +123,15 @@ bsrng_t* bsrng_create_ex(bsrng_cipher cipher, const uint8_t* keys, const uint8_t
 /*
  * bsrng_rekey -- re-initialise every instance of an existing handle with new
  * keys/IVs (same n, iv_bits): slice + initialisation clocks into the handle's
- * state, resetting its bit counter.  Asynchronous on `stream` (host inputs
- * are staged through a pinned buffer, so the caller may reuse them on return).
+ * state, resetting its bit counter.  Asynchronous on `stream`: no host
+ * synchronisation (AES: the key expansion runs on the device and its round
+ * keys reach the handle's constant-memory slot by a stream-ordered copy).
+ * Host inputs (BSRNG_INPUT_HOST) are copied into a handle-owned pinned buffer
+ * before the call returns, so the caller may overwrite them immediately (the
+ * call waits only for the previous rekey's copy out of that buffer).  Device
+ * inputs (BSRNG_INPUT_DEVICE) must stay valid until `stream` passes the call.
+ * Errors: EINVAL (NULL, unknown flags, a stream of another device), ENOMEM,
+ * ECUDA.
  */
 int bsrng_rekey(bsrng_t* h, const uint8_t* keys, const uint8_t* ivs, uint32_t flags,
                 void* stream);
@@ -121,17 +142,22 @@ int bsrng_rekey(bsrng_t* h, const uint8_t* keys, const uint8_t* ivs, uint32_t fl
  * `layout`.  Asynchronous on `stream`.
  *   out  : DEVICE memory, caller-owned, bsrng_out_bytes(h, bits, layout) bytes,
  *          16-byte aligned (CHECKSUM: 8-byte aligned; it is overwritten).
- *   bits_per_instance: multiple of 32 (AES: of 128); 0 is a no-op.
- * Errors: EINVAL (NULL, alignment, bits, layout), ERANGE (cumulative bits per
- * instance > 2^40), ECUDA.
+ *   bits_per_instance: multiple of 32 (AES: of 128); 0 is a no-op.  Calls of
+ *          more than 2^31 bits per instance run as several time segments of
+ *          one launch (the same result as one pass).
+ *   stream: must belong to the handle's device (else EINVAL); NULL = the
+ *          legacy default stream.
+ * Errors: EINVAL (NULL, alignment, bits, layout, stream), ERANGE (cumulative
+ * bits per instance above the cipher's limit, see BSRNG_ERANGE), ECUDA.
  */
 int bsrng_generate(bsrng_t* h, void* out, uint64_t bits_per_instance, bsrng_layout layout,
                    void* stream);
 
 /*
  * bsrng_generate_host -- as bsrng_generate but `host_out` is HOST memory of
- * bsrng_out_bytes bytes; the data is produced on the device in chunks and
- * copied back; synchronises `stream` before returning.
+ * bsrng_out_bytes bytes (any alignment); the data is produced on the device in
+ * chunks of at most 1 GiB (a handle-owned device bounce buffer) and copied
+ * back; synchronises `stream` before returning.  CHECKSUM: 8 bytes.
  */
 int bsrng_generate_host(bsrng_t* h, void* host_out, uint64_t bits_per_instance,
                         bsrng_layout layout, void* stream);
@@ -157,20 +183,15 @@ int64_t bsrng_copy_state(const bsrng_t* h, uint32_t* host_out, uint64_t words);
 
 /*
  * bsrng_set_option -- tuning knobs (for sweeps; defaults are the tuned ones).
- *   "block"      : threads per block for the keystream kernel (multiple of 32)
- *   "sched"      : 0 = one thread per group for the whole call,
- *                  1 = persistent, time-segmented work queue (default)
- *   "seg_clocks" : clocks per work item when sched = 1 (multiple of 32)
- *   "ctas_per_sm": resident CTAs per SM for the persistent grid
- *   "unroll"     : clocks per loop iteration (MICKEY 2, 4, 8; Grain 8, 16, 32)
+ *   "sched"      : 0 = one thread per group for the whole call (calls of more
+ *                  than 2^31 bits still use the queue), 1 = persistent,
+ *                  time-segmented work queue (default)
+ *   "seg_clocks" : clocks per work item when sched = 1 (multiple of 32; 0 = auto)
+ *   "ctas_per_sm": resident CTAs per SM for the persistent grid (0 = auto)
+ *   "unroll"     : clocks per loop iteration: Grain / LFSR 32 (default) or 16;
+ *                  MICKEY 4 (the only one built); 0 = default
  *   "rm_ws"      : ROW_MAJOR kernel: -1 auto, 1 warp-specialised (AES: block-
  *                  lane), 0 plain
- *   "rm_slots"   : ROW_MAJOR plain kernel: 32-clock blocks staged per row
- *                  before a flush, 8 (one 32 B sector per row) or 4 (16 B,
- *                  half the shared memory); 0 = auto
- *   "rm_zreg"    : ROW_MAJOR plain kernel with 32 clocks per iteration: keep
- *                  the z block in registers (1, default) or stage it in
- *                  shared memory (0)
  *   "rm_tmem"    : ROW_MAJOR plain kernel: stage the row segments in tensor
  *                  memory (TMEM, 256 columns per CTA, two CTAs per SM) (1)
  *                  or in shared memory (0); -1 = cipher default (MICKEY /
@@ -178,13 +199,13 @@ int64_t bsrng_copy_state(const bsrng_t* h, uint32_t* host_out, uint64_t words);
  *   "rm_tma"     : TMEM staging: whole-sector flushes of warps whose rows are
  *                  all real as TMA tensor stores when the row stride is a
  *                  multiple of 16 B (1, default) or as 8 B stores (0)
- *   "rm_dbl"     : TMEM staging with one CTA per SM and one work item per
- *                  warp-unit: double-buffered staging (512 columns), the
- *                  previous sector period flushed 4 rows per block (1,
- *                  default) or a single buffer (0)
- *   "init_fused" : MICKEY / Grain create/rekey: slicing fused into the
- *                  initialisation kernel (1, default) or the separate
- *                  slice_bits + preclock kernels (0)
+ *   "rm_dbl"     : TMEM staging with one CTA per SM and one time segment:
+ *                  double-buffered staging (512 columns), the previous sector
+ *                  period flushed 4 rows per block (1, default) or a single
+ *                  buffer (0)
+ *   "init_fused" : create/rekey: slicing fused into the initialisation kernel
+ *                  (1, default) or the separate ballot slice (+ preclock)
+ *                  kernels (0)
  * Returns BSRNG_OK or BSRNG_EINVAL for an unknown key/value.
  */
 int bsrng_set_option(bsrng_t* h, const char* key, int64_t value);

@@ -183,7 +183,9 @@ class Generator:
         kp, kdev = _ptr(keys)
         if ivs is not None and getattr(ivs, "size", 1) == 0:
             ivs = None
-        vp, _ = _ptr(ivs)
+        vp, vdev = _ptr(ivs)
+        if ivs is not None and vdev != kdev:
+            raise ValueError("keys and ivs must both be host or both be device buffers")
         self._keep = (keys, ivs)
         _check(lib().bsrng_rekey(self._h, kp, vp, INPUT_DEVICE if kdev else INPUT_HOST,
                                  _stream_ptr(stream)))

@@ -39,6 +39,15 @@ struct RoundKeys {
     uint32_t m[11][128];
 };
 
+// Round keys live in constant memory, one slot per AES handle: the key
+// expansion kernel writes the masks to device memory and a stream-ordered
+// device-to-device cudaMemcpyToSymbolAsync moves them into the handle's slot,
+// so a rekey never waits on the host.  The keystream kernels read them with a
+// warp-uniform (slot, round) index -- uniform constant loads (LDCU) feeding
+// the AddRoundKey LOP3s.  11 slots x 5.5 KB fit the 64 KB constant bank.
+constexpr int RK_SLOTS = 11;
+__constant__ RoundKeys c_rk[RK_SLOTS];
+
 // AES S-box on one byte held MSB-first in 8 slice words (in place): the
 // Boyar-Peralta depth-16 circuit (113 two-input gates) mapped onto 84
 // three-input LOP3s by tools/lut3_map.py (cut enumeration + area recovery),
@@ -271,8 +280,9 @@ __global__ void __launch_bounds__(32) aes_key_expand_kernel(const uint8_t* __res
 //              (two encryptions fill a sector) and written as 16 B stores.
 // ---------------------------------------------------------------------------
 template <int LAYOUT>
-__global__ void __launch_bounds__(128, 2) aes_ctr_kernel(const KsArgs a, const __grid_constant__ aes::RoundKeys rk)
+__global__ void __launch_bounds__(128, 2) aes_ctr_kernel(const __grid_constant__ KsArgs a, int rk_slot)
 {
+    const aes::RoundKeys& rk = aes::c_rk[rk_slot];
     constexpr int NW = 4;
     extern __shared__ uint32_t aes_smem[];  // base counters [128][128 threads] (+ ROW_MAJOR sector buffers)
     __shared__ uint32_t s_item[NW];
@@ -384,11 +394,13 @@ __global__ void __launch_bounds__(128, 2) aes_ctr_kernel(const KsArgs a, const _
 // encryption -- whole sectors with no shared-memory staging.  Used when a call
 // has >= 32 blocks per instance (otherwise most lanes would be wasted).
 // Work items: (time segment of whole 4096-bit encryptions, 32-instance warp);
-// `a.units` counts warps here, `a.aux` = row-major initial counters (n x 16 B).
+// `a.units` counts warps here.  A warp's 32 instances are group w, so each
+// thread reads its initial counter back out of the group's sliced state rows
+// (bit `lane` of row b = FIPS bit b of its counter block).
 // ---------------------------------------------------------------------------
-__global__ void __launch_bounds__(128, 2) aes_ctr_rowmajor_lanes_kernel(const KsArgs a,
-                                                                         const __grid_constant__ aes::RoundKeys rk)
+__global__ void __launch_bounds__(128, 2) aes_ctr_rowmajor_lanes_kernel(const __grid_constant__ KsArgs a, int rk_slot)
 {
+    const aes::RoundKeys& rk = aes::c_rk[rk_slot];
     __shared__ uint32_t s_item[4];
     volatile uint32_t* slot = s_item + (threadIdx.x >> 5);
     next_item(a, slot);
@@ -414,14 +426,14 @@ __global__ void __launch_bounds__(128, 2) aes_ctr_rowmajor_lanes_kernel(const Ks
         const uint64_t bit_begin = seg * a.seg_clocks;
         const uint64_t left = a.nclocks - bit_begin;
         const uint64_t nblocks = (left < a.seg_clocks ? left : a.seg_clocks) >> 7;
-        // V = ctr_inst + first block index of this item (128-bit big-endian)
+        // V = ctr_inst + first block index of this item (128-bit big-endian),
+        // the counter gathered from the sliced state (warp-uniform addresses)
         uint32_t V[4] = {0, 0, 0, 0};
-        if (real) {
-            const uint8_t* cb = static_cast<const uint8_t*>(a.aux) + inst * 16;
+        {
+            const uint32_t* src = opaque(a.state + w);
 #pragma unroll
-            for (int k = 0; k < 4; ++k)
-                V[k] = (uint32_t(cb[4 * k]) << 24) | (uint32_t(cb[4 * k + 1]) << 16) | (uint32_t(cb[4 * k + 2]) << 8) |
-                       uint32_t(cb[4 * k + 3]);
+            for (int b = 0; b < 128; ++b)
+                V[b >> 5] |= ((__ldcg(src + uint64_t(b) * a.Gp) >> lane) & 1u) << (31 - (b & 31));
         }
         {
             const uint64_t T = (a.t0 + bit_begin) >> 7;

@@ -118,7 +118,8 @@ struct Grain {
     // clocks per loop iteration (~45 instructions per clock).  The 80-clock
     // register rotation costs 160/U moves per clock at the back edge; at U = 32
     // ptxas emits them all as IMAD.MOV (FMA pipe), at U = 16 partly as MOV.
-    static constexpr int U_DEFAULT = 32, U_ALT0 = 8, U_ALT1 = 16;
+    // (U = 8 was dropped after the round-1 sweep: 0.83 of roofline)
+    static constexpr int U_DEFAULT = 32, U_ALT0 = 16, U_ALT1 = 16;
     // ROW_MAJOR default: row segments staged in TMEM, two CTAs per SM (+7%
     // over one CTA with smem staging; DESIGN.md sec. 5 Grain)
     static constexpr bool RM_TMEM = true;

@@ -122,7 +122,6 @@ struct KsArgs {
     uint32_t* ticket;     // persistent mode: [1], zeroed before launch
     uint32_t* flags;      // persistent mode: [units], zeroed before launch
     uint32_t* scratch;    // [32] sink for padding-group SLICED stores
-    const void* aux;      // cipher-specific input (AES block-lane ROW_MAJOR: counters)
     unsigned long long* dbg;  // optional scheduler counters (BSRNG_DEBUG), or null
     int persistent;
     // ROW_MAJOR + TMEM: whole-sector flushes of warps whose 32 groups are all

@@ -20,7 +20,7 @@ namespace bsk {
 struct Lfsr128 {
     static constexpr int NSTATE = 128;
     static constexpr bool MSB_FIRST = true;
-    static constexpr int U_DEFAULT = 32, U_ALT0 = 8, U_ALT1 = 16;
+    static constexpr int U_DEFAULT = 32, U_ALT0 = 16, U_ALT1 = 16;
     static constexpr bool RM_TMEM = false, RM_SEGMENTED = true;
     // consume: one 128-clock body (the rotation period), no moves (keystream.cuh)
     static constexpr int U_CONSUME = 128;

@@ -319,8 +319,10 @@ struct Mickey2 {
     static constexpr int NSTATE = m2::NSTATE;
     static constexpr bool MSB_FIRST = true;  // spec [5]: keystream packed MSB-first
     // clocks per loop iteration: 4 keeps the loop (21 KB of SASS) in the
-    // instruction cache; 2 and 8 are built for sweeps ("unroll" option)
-    static constexpr int U_DEFAULT = 4, U_ALT0 = 2, U_ALT1 = 8;
+    // instruction cache.  Only U = 4 is built: U = 8 overflowed the cache
+    // (0.92 of roofline, 270 B of stack) and at U = 2 ptxas put the whole
+    // consume state in local memory (round-1 sweep).
+    static constexpr int U_DEFAULT = 4, U_ALT0 = 4, U_ALT1 = 4;
     // ROW_MAJOR default: the plain clock kernel with row segments staged in
     // TMEM, two CTAs per SM, one work item per warp-unit (0.935 of the ALU
     // roofline vs 0.904 for the smem warp-specialised kernel)
@@ -389,35 +391,24 @@ __global__ void __launch_bounds__(128) m2_preclock_kernel(const uint32_t* __rest
     uint32_t r[100], s[100];
 #pragma unroll
     for (int i = 0; i < 100; ++i) r[i] = s[i] = 0u;
-    // 4 clocks per loop iteration (iv_bits is a multiple of 8): the S-register
-    // renaming then closes inside the body instead of costing ~100 moves/clock.
-    // The input words of the next 4 clocks are loaded one iteration ahead, so
-    // their HBM latency hides behind ~1300 LOP3 (ncu: long-scoreboard was the
-    // second stall reason without the prefetch).
-    const int nin = iv_bits + 80;
+    // The spec's input sequence is iv_bits IV bits, 80 key bits, then 100
+    // zero bits: T = iv_bits + 180 mixing clocks, 4 per loop iteration (the
+    // S-register renaming closes inside the body), then the last T mod 4
+    // (< 100, so zero-input) clocks one at a time -- any iv_bits in 0..80.
+    const int nin = iv_bits + 80, T = nin + 100, T4 = T & ~3;
     const uint32_t* iv_p = iv_s + g;
     const uint32_t* key_p = key_s + g - uint64_t(iv_bits) * Gp;
-    auto in_ptr = [&](int c) { return (c < iv_bits ? iv_p : key_p) + uint64_t(c) * Gp; };
-    uint32_t cur[4];
-#pragma unroll
-    for (int u = 0; u < 4; ++u) cur[u] = __ldcs(in_ptr(u));
+    auto in_word = [&](int c) { return c < nin ? __ldcs((c < iv_bits ? iv_p : key_p) + uint64_t(c) * Gp) : 0u; };
 #pragma unroll 1
-    for (int c = 0; c < nin; c += 4) {
-        uint32_t nxt[4] = {0u, 0u, 0u, 0u};
-        if (c + 4 < nin) {
+    for (int c = 0; c < T4; c += 4) {
+        uint32_t in[4];
 #pragma unroll
-            for (int u = 0; u < 4; ++u) nxt[u] = __ldcs(in_ptr(c + 4 + u));
-        }
+        for (int u = 0; u < 4; ++u) in[u] = in_word(c + u);
 #pragma unroll
-        for (int u = 0; u < 4; ++u) m2::clock_kg<true>(r, s, cur[u]);
-#pragma unroll
-        for (int u = 0; u < 4; ++u) cur[u] = nxt[u];
+        for (int u = 0; u < 4; ++u) m2::clock_kg<true>(r, s, in[u]);
     }
 #pragma unroll 1
-    for (int i = 0; i < 100; i += 4) {
-#pragma unroll
-        for (int u = 0; u < 4; ++u) m2::clock_kg<true>(r, s, 0u);
-    }
+    for (int c = T4; c < T; ++c) m2::clock_kg<true>(r, s, 0u);
 #pragma unroll
     for (int i = 0; i < 100; ++i) state[uint64_t(i) * Gp + g] = r[i];
 #pragma unroll
@@ -468,22 +459,24 @@ __global__ void __launch_bounds__(M2I_BLOCK, 2) m2_init_kernel(const uint8_t* __
     uint32_t r[m2::RN], s[100];
 #pragma unroll
     for (int i = 0; i < 100; ++i) r[i] = s[i] = 0u;
-    const int nin = iv_bits + 80;  // IV clocks, then key clocks: rows 0..iv_bits-1, 80..159
+    // T = iv_bits + 180 mixing clocks: IV bits (rows 0..iv_bits-1), key bits
+    // (rows 80..159), 100 zero bits; 4-clock deferred-reduction blocks, then
+    // the last T mod 4 (zero-input) clocks in Galois form, so any iv_bits in
+    // 0..80 works (the block loop needs whole 4-clock blocks)
+    const int nin = iv_bits + 80, T = nin + 100, T4 = T & ~3;
 #pragma unroll 1
-    for (int c = 0; c < nin; c += 4) {
+    for (int c = 0; c < T4; c += 4) {
         uint32_t in[4];
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
-            const int row = c + u < iv_bits ? c + u : c + u - iv_bits + 80;
-            in[u] = sl[row * M2I_BLOCK];
+            const int cu = c + u;
+            const int row = cu < iv_bits ? cu : cu - iv_bits + 80;
+            in[u] = cu < nin ? sl[row * M2I_BLOCK] : 0u;
         }
         m2::clock4_mix(r, s, in);
     }
 #pragma unroll 1
-    for (int i = 0; i < 100; i += 4) {
-        const uint32_t in[4] = {0u, 0u, 0u, 0u};
-        m2::clock4_mix(r, s, in);
-    }
+    for (int c = T4; c < T; ++c) m2::clock_kg<true>(r, s, 0u);
     uint32_t* p = opaque(state + g);
 #pragma unroll
     for (int i = 0; i < 100; ++i) __stcg(p + uint64_t(i) * Gp, r[i]);

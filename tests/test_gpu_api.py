@@ -49,15 +49,14 @@ def test_zero_bits_is_noop(cipher):
 
 
 @pytest.mark.parametrize("cipher,opts", [
-    ("mickey2", {"unroll": 2}), ("mickey2", {"unroll": 8}), ("mickey2", {"sched": 0}),
+    ("mickey2", {"unroll": 4}), ("mickey2", {"sched": 0}),
     ("mickey2", {"ctas_per_sm": 2}), ("mickey2", {"rm_ws": 0}), ("mickey2", {"rm_ws": 1, "seg_clocks": 512}),
     ("mickey2", {"rm_ws": 1}), ("mickey2", {"rm_tmem": 0}), ("mickey2", {"rm_tmem": 1, "seg_clocks": 384}),
-    ("grain", {"unroll": 8}), ("grain", {"unroll": 16}), ("grain", {"rm_ws": 1}), ("grain", {"sched": 0}),
+    ("grain", {"unroll": 16}), ("grain", {"rm_ws": 1}), ("grain", {"sched": 0}),
     ("grain", {"ctas_per_sm": 1, "seg_clocks": 256}),
-    ("grain", {"rm_tmem": 0}), ("grain", {"rm_tmem": 0, "rm_slots": 4, "rm_zreg": 0}),
-    ("grain", {"rm_tmem": 0, "rm_slots": 8, "rm_zreg": 0}),
-    ("grain", {"rm_tmem": 0, "rm_slots": 4, "ctas_per_sm": 2, "seg_clocks": 384}),
-    ("mickey2", {"rm_ws": 0, "rm_slots": 4}), ("mickey2", {"rm_ws": 0, "rm_slots": 4, "seg_clocks": 160}),
+    ("grain", {"rm_tmem": 0}), ("grain", {"rm_tmem": 0, "unroll": 16}),
+    ("grain", {"rm_tmem": 0, "ctas_per_sm": 2, "seg_clocks": 384}),
+    ("mickey2", {"rm_ws": 0, "rm_tmem": 0}), ("mickey2", {"rm_ws": 0, "rm_tmem": 0, "seg_clocks": 160}),
     ("aes128ctr", {"ctas_per_sm": 1}), ("aes128ctr", {"rm_ws": 0}), ("aes128ctr", {"seg_clocks": 4096}),
 ])
 def test_options_stay_bit_exact(cipher, opts):
@@ -81,8 +80,8 @@ def test_options_stay_bit_exact(cipher, opts):
 def test_option_validation():
     keys, ivs = inputs.make_inputs("grain", 32)
     g = bsrng.Generator("grain", keys, ivs)
-    for k, v in (("unroll", 4), ("sched", 2), ("seg_clocks", 33), ("ctas_per_sm", 99), ("rm_ws", 5),
-                 ("rm_slots", 2), ("rm_zreg", 3), ("rm_tmem", 2), ("init_fused", 2)):
+    for k, v in (("unroll", 4), ("unroll", 8), ("sched", 2), ("seg_clocks", 33), ("ctas_per_sm", 99), ("rm_ws", 5),
+                 ("rm_slots", 4), ("rm_zreg", 0), ("rm_tmem", 2), ("rm_tma", 2), ("rm_dbl", 2), ("init_fused", 2)):
         with pytest.raises(bsrng.BsrngError) as e:
             g.set_option(k, v)
         assert e.value.code == bsrng.EINVAL
@@ -136,7 +135,6 @@ def test_mickey_2_40_limit_boundary():
     ("grain", {"rm_tmem": 1}, 8192),
     ("grain", {"rm_tmem": 1}, 4416),                      # 552 B rows: 8 B-aligned flushes
     ("grain", {"rm_tmem": 1, "seg_clocks": 160}, 2080),   # partial slots at segment ends
-    ("grain", {"rm_tmem": 1, "rm_zreg": 0}, 8192),
     ("grain", {"rm_tmem": 1, "unroll": 16}, 4128),
     ("grain", {"rm_tmem": 1, "sched": 0}, 2048),
     ("grain", {"rm_tmem": 1, "ctas_per_sm": 2, "seg_clocks": 512}, 4096),

@@ -36,7 +36,7 @@ def test_spec_vectors_on_gpu(row):
     assert got.startswith(ks)
 
 
-@pytest.mark.parametrize("unroll", [0, 8, 16])
+@pytest.mark.parametrize("unroll", [0, 16])
 def test_ragged_all_layouts(unroll):
     n, bits = 32 * 37 + 13, 2048
     keys, ivs = inputs.make_inputs("grain", n)
