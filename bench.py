@@ -34,15 +34,21 @@ sys.path.insert(0, ROOT)
 
 N_DEFAULT = 1 << 22
 BITS_DEFAULT = 1 << 20
-# Algorithmic LOP3 per keystream bit position per 32-instance group (DESIGN.md
-# sec. 5): MICKEY 2.0 327 per clock in the spec's Galois form (SURVEY App. D,
-# output op included), 304 with the R reduction deferred over K = 4-clock
-# blocks (315.5 at K = 2; mickey2.cuh clock_lazy, DESIGN.md sec. 5 item 10);
-# Grain v1 37 per clock (f 3 + g 25 + h/z 9) + 1 to fold into the checksum;
-# AES-128-CTR 17280 per 32-block encryption (4096 bit positions) + 64 for the
-# checksum XOR tree.
+# LOP3 per keystream bit position per 32-instance group (one clock of one
+# thread).  Two counts per cipher:
+#  * ALGORITHMIC -- SURVEY.md sec. 8(d)'s per-unit figure, the roofline
+#    numerator the contract fixes: MICKEY 2.0 327 per clock (the spec's Galois
+#    form, output op included), Grain v1 39 (App. D's
+#    decomposition), AES-128-CTR 17280 per 32-block encryption (4096 bit
+#    positions; DESIGN.md sec. 5 AES), the LFSR's Eq. 2 feedback 2 (k = 4 taps).
+#  * KERNEL -- what the shipped kernels need: MICKEY 304 with the R reduction
+#    deferred over K = 4-clock blocks (315.5 at K = 2; mickey2.cuh clock_lazy,
+#    DESIGN.md sec. 5 item 10), Grain 37 (+1 to fold into the checksum), AES
+#    17280 (+64 for the checksum XOR tree), LFSR 2 (+0.5 for the checksum).
+# A kernel whose count is below the algorithmic one can exceed frac = 1.
 MICKEY2_GALOIS_OPS = 327.0
 MICKEY2_OPS_BY_BLOCK = {1: 327.0, 2: 315.5, 4: 304.0}
+ALGORITHMIC_OPS = {"mickey2": 327.0, "grain": 39.0, "aes128ctr": 17280.0 / 128.0, "lfsr128": 2.0}
 
 
 def mickey2_block(unroll):
@@ -51,15 +57,18 @@ def mickey2_block(unroll):
 
 
 def lop3_per_bit(cipher, mode, unroll=None):
+    """KERNEL count (see above) per clock per 32-instance group."""
     if cipher == "mickey2":
         return MICKEY2_OPS_BY_BLOCK[mickey2_block(unroll or 4)]
     if cipher == "grain":
         return 38.0 if mode == "consume" else 37.0
     if cipher == "lfsr128":
-        # feedback XOR4 = 2 LOP3; consume folds two clocks' output words into
-        # the accumulator with one XOR3 (0.5 per clock; 128-clock loop body)
+        # feedback XOR4 = 2 LOP3; consume folds the period's output words into
+        # the accumulator (0.5 per clock; 128-clock loop body)
         return 2.5 if mode == "consume" else 2.0
     return (17280.0 + (64.0 if mode == "consume" else 0.0)) / 128.0
+
+
 CIPHER_NAME = {"mickey2": "MICKEY 2.0", "grain": "Grain v1", "aes128ctr": "AES-128-CTR",
                "lfsr128": "bitsliced LFSR-128 (Eq. 2)"}
 ALU_LANES_PER_SM_CLK = 64      # 4 SMSP x 16 lanes (alu pipe rt = 2 cycles/warp-instr)
@@ -83,7 +92,9 @@ def parse():
                         "c4 = configs[3]: the paper's launch shape, 2^19 instances x 4416 clocks per GPU; "
                         "rekey = SURVEY NEXT-3: 2^22 short streams x 2^10 bits, key/IV setup dominates")
     p.add_argument("--cipher", default="mickey2", choices=["mickey2", "grain", "aes128ctr", "lfsr128"])
-    p.add_argument("--n", type=int, default=None, help="instances per GPU (c2) / in total (c3)")
+    p.add_argument("--instances", "--n", dest="n", type=int, default=None,
+                   help="instances per GPU (c2/c4/rekey) / in total (c3); use --instances under torchrun "
+                        "(its parser takes --n for one of its own options)")
     p.add_argument("--bits", type=int, default=None, help="keystream bits per instance per step")
     p.add_argument("--no-context", action="store_true", help="skip the ALU-peak / cuRAND microbenchmarks")
     p.add_argument("--mode", default="consume", choices=["consume", "materialise"],
@@ -97,6 +108,10 @@ def parse():
     p.add_argument("--ctas-per-sm", type=int, default=None)
     p.add_argument("--opt", action="append", default=[], metavar="KEY=VALUE",
                    help="extra bsrng_set_option knob (A/B runs; defaults are the tuned ones)")
+    p.add_argument("--test-delay-rank", type=int, default=-1, help=argparse.SUPPRESS)  # tests: MAX over ranks
+    p.add_argument("--backend", default=os.environ.get("BSRNG_DIST_BACKEND", "nccl"), choices=["nccl", "gloo"],
+                   help="process-group backend for N > 1 (gloo lets two ranks share one GPU in tests; "
+                        "only the max step time and the checksum cross ranks)")
     return p.parse_args()
 
 
@@ -116,7 +131,7 @@ class ClockSampler:
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
-                 "-lms", "200"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+                 "-lms", "50"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
         except FileNotFoundError:
@@ -174,7 +189,7 @@ def profile_traffic():
 TRAFFIC_CAPTURE = {("mickey2", "consume"): "ks_consume", ("mickey2", "materialise"): "ks_rowmajor",
                    ("grain", "consume"): "grain_consume", ("grain", "materialise"): "grain_rowmajor",
                    ("aes128ctr", "consume"): "aes_consume", ("aes128ctr", "materialise"): "aes_rowmajor",
-                   ("lfsr128", "materialise"): "lfsr_sliced"}
+                   ("lfsr128", "consume"): "lfsr_consume", ("lfsr128", "materialise"): "lfsr_rowmajor"}
 
 
 def traffic_for(cipher, mode, n, launch_bits):
@@ -256,15 +271,18 @@ def cpu_baseline(target_s=25.0, cipher="mickey2"):
             "bits_per_s_per_core": r / cores}
 
 
-def run_context(local_rank):
-    """Live context numbers on this GPU: the measured LOP3 issue ceiling,
-    cuRAND on the same B200 and the HBM write-only bandwidth (STG.128 /
-    STG.32 streams; tools/microbench, built by __graft_entry__.build)."""
+def run_context(local_rank, names=("alu_peak", "curand", "write_peak")):
+    """Live context numbers on this GPU: the measured LOP3 issue ceiling (the
+    roofline denominator, measured before the timed region), cuRAND on the
+    same B200 and the HBM write-only bandwidth (STG.128 / STG.32 streams;
+    tools/microbench, built by __graft_entry__.build)."""
     out = {}
     mb = os.path.join(ROOT, "tools", "microbench")
     env = dict(os.environ, CUDA_VISIBLE_DEVICES=os.environ.get("CUDA_VISIBLE_DEVICES", str(local_rank)))
     exes = {"alu_peak": "alu_peak", "curand": "curand_bench", "write_peak": "write_peak"}
-    for name, argv in (("alu_peak", ["200000"]), ("curand", ["4294967296"]), ("write_peak", [])):
+    argvs = {"alu_peak": ["200000"], "curand": ["4294967296"], "write_peak": []}
+    for name in names:
+        argv = argvs[name]
         exe = os.path.join(mb, exes[name])
         if not os.path.exists(exe):
             out[name] = "not built"
@@ -341,14 +359,19 @@ def run_ours(args, rank, world, local_rank):
 
     from paper_conf_icppw_monfaredhkzrg20_b200 import shard
 
-    dev = torch.device("cuda", local_rank)
+    # one rank per GPU; with --backend gloo two ranks may share a GPU (tests)
+    dev = torch.device("cuda", local_rank % torch.cuda.device_count())
     torch.cuda.set_device(dev)
+    coll_dev = dev if (world > 1 and args.backend == "nccl") else None  # gloo reduces CPU tensors
     n_total, bits, scaling, desc = workload(args, world)
     if args.workload in ("c2", "c4", "rekey"):
         first, n = shard.weak_range(rank, n_total // world)
     else:
         first, n = shard.strong_range(rank, world, n_total)
     stream = torch.cuda.Stream(dev)
+
+    # the measured LOP3 issue ceiling on this GPU (roofline denominator)
+    peak_ctx = run_context(dev.index, ("alu_peak",)) if rank == 0 and not args.no_context else {}
 
     keys_h, ivs_h = inputs.make_inputs(args.cipher, n, first)
     if args.cipher == "aes128ctr":
@@ -373,9 +396,15 @@ def run_ours(args, rank, world, local_rank):
         if world > 1:
             dist.barrier()
 
+    def delay():  # test hook (--test-delay-rank): ~50 ms more on one rank
+        if rank == args.test_delay_rank:
+            with torch.cuda.stream(stream):
+                torch.cuda._sleep(100_000_000)
+
     def step_consume(ev=None):
         if ev:
             ev[2].record(stream)
+        delay()
         g.rekey(keys_d, ivs_d, stream=stream)
         if ev:
             ev[0].record(stream)
@@ -425,53 +454,64 @@ def run_ours(args, rank, world, local_rank):
             rekey_ms.append(r0.elapsed_time(k0))
         clocks = sampler.stop() if sampler else None
         launches = bsrng.launch_count() - l0
-        t = torch.tensor([sum(step_ms), sum(kern_ms), sum(rekey_ms)], dtype=torch.float64, device=dev)
-        if world > 1:
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        timed.rekey_ms = float(t[2]) / steps
-        return float(t[0]) / steps, float(t[1]) / steps, launches, clocks
+        # MAX over ranks of each rank's summed step / kernel / rekey times
+        t = [shard.allreduce_max(sum(x), device=coll_dev) for x in (step_ms, kern_ms, rekey_ms)]
+        timed.rekey_ms = t[2] / steps
+        timed.rank_ms = sum(step_ms) / steps
+        return t[0] / steps, t[1] / steps, launches, clocks
 
     peaks = measured_peaks()
     sm_max = float(peaks.get("sm_max_mhz", 1965.0))
     nsm = torch.cuda.get_device_properties(dev).multi_processor_count
+    derived_peak = nsm * ALU_LANES_PER_SM_CLK * sm_max * 1e6 / 1e12
+    measured_peak = peak_ctx.get("alu_peak_tlop3_per_s")
 
     def init_roofline(rk_ms):
         """a-1 + a-2 (bsrng_rekey) against the same ALU peak: initialisation
         clocks x ops per clock (MICKEY 260 x 306 with the deferred R reduction
         -- 328 in Galois form: 304 - 1 output + u = INPUT_BIT ^ s50 + its XOR
         into the pending word + FEEDBACK_S --, Grain 160 x 39; AES-CTR has no
-        initialisation clocks, only slicing + a one-thread key expansion)."""
+        initialisation clocks, only slicing + a one-warp key expansion)."""
         ops = {"mickey2": 260 * 306.0, "grain": 160 * 39.0}.get(args.cipher)
         if not ops or rk_ms <= 0:
             return None
         achieved = ops * (n // 32) / (rk_ms * 1e-3) / 1e12
-        peak = nsm * ALU_LANES_PER_SM_CLK * sm_max * 1e6 / 1e12
-        return {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TLOP3/s", "frac": achieved / peak,
-                "note": "rekey = slice kernels + preclock kernel (+ H2D for e2e)"}
+        return {"bound": "alu", "achieved": achieved, "peak": derived_peak, "unit": "TLOP3/s",
+                "frac": achieved / derived_peak, "note": "rekey = fused slicing + initialisation kernel"}
 
     def roofline(kern_ms_per_step, clocks, mode):
+        """achieved = ALGORITHMIC LOP3 (the sec. 8(d) per-clock
+        count x groups x clocks) / the keystream kernel's CUDA-event time,
+        against the LOP3 ceiling measured in this run (tools/microbench/alu_peak,
+        before the timed region); the derived 148 x 64 lanes x sm_max peak and
+        the kernel's own op count are reported beside it."""
         unroll = dict(kv.split("=", 1) for kv in args.opt).get("unroll")
-        ops = lop3_per_bit(args.cipher, mode, int(unroll) if unroll else None)
-        lop3 = ops * (n // 32) * bits  # algorithmic LOP3 per step, dominant kernel
-        achieved = lop3 / (kern_ms_per_step * 1e-3) / 1e12
-        peak = nsm * ALU_LANES_PER_SM_CLK * sm_max * 1e6 / 1e12
-        out = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TLOP3/s", "frac": achieved / peak,
-               "peak_basis": f"{nsm} SMs x {ALU_LANES_PER_SM_CLK} LOP3 lanes/clk x sm_max {sm_max:.0f} MHz "
-                             "(B300_MICROARCH alu pipe rt=2/SMSP; DESIGN.md)",
+        alg = ALGORITHMIC_OPS[args.cipher]
+        kops = lop3_per_bit(args.cipher, mode, int(unroll) if unroll else None)
+        units = (n // 32) * bits / (kern_ms_per_step * 1e-3) / 1e12  # group-clocks per s, x 1e12
+        peak = measured_peak or derived_peak
+        out = {"bound": "alu", "achieved": alg * units, "peak": peak, "unit": "TLOP3/s",
+               "frac": alg * units / peak,
+               "peak_basis": ("measured in this run: tools/microbench/alu_peak (independent lop3.b32 chains on "
+                              "every SM)" if measured_peak else
+                              f"derived: {nsm} SMs x {ALU_LANES_PER_SM_CLK} LOP3 lanes/clk x sm_max {sm_max:.0f} "
+                              "MHz (alu_peak not run)"),
+               "ops_per_clock_algorithmic": alg,
+               "ops_per_clock_basis": "SURVEY.md sec. 8(d) / App. D per-clock LOP3 count",
+               "ops_per_clock_kernel": kops,
+               "frac_kernel_ops": kops * units / peak,
+               "peak_derived": derived_peak,
+               "frac_vs_derived_peak": alg * units / derived_peak,
                "traffic": None}
-        if args.cipher == "mickey2":
-            out["ops_per_clock"] = ops
-            out["galois_ops_per_clock"] = MICKEY2_GALOIS_OPS
-            out["frac_vs_galois_count"] = out["frac"] * MICKEY2_GALOIS_OPS / ops
         if clocks and clocks.get("sm_mhz"):
-            out["frac_at_sampled_clock"] = achieved / (nsm * ALU_LANES_PER_SM_CLK * clocks["sm_mhz"] * 1e6 / 1e12)
+            out["frac_at_sampled_clock"] = alg * units / (nsm * ALU_LANES_PER_SM_CLK * clocks["sm_mhz"] * 1e6 / 1e12)
         return out
 
     results = {}
     modes = [args.mode] + ([] if args.no_other_mode else [m for m in ("consume", "materialise") if m != args.mode])
     for mode in modes:
         fn = step_consume if mode == "consume" else step_materialise
-        sampler = ClockSampler(local_rank) if (rank == 0 and mode == args.mode) else None
+        sampler = ClockSampler(dev.index) if rank == 0 else None
         ms, kms, launches, clocks = timed(fn, args.steps, args.warmup, sampler)
         tbps = n_total * bits / (ms * 1e-3) / 1e12
         rk_ms = timed.rekey_ms
@@ -480,6 +520,8 @@ def run_ours(args, rank, world, local_rank):
                "preclock_roofline": init_roofline(rk_ms),
                "kernel_tbps_per_gpu": n * bits / (kms * 1e-3) / 1e12,
                "gpu_launches": launches, "roofline": roofline(kms, clocks, mode)}
+        if world > 1:
+            res["rank0_ms_per_step"] = timed.rank_ms
         if mode == "materialise":
             out_bytes = n * bits / 8
             res["hbm_write_gbs_per_gpu"] = out_bytes / (kms * 1e-3) / 1e9
@@ -492,36 +534,40 @@ def run_ours(args, rank, world, local_rank):
     # checksum of one consume step (sharding invariant), outside the timed region
     step_consume()
     torch.cuda.synchronize(dev)
-    checksum = shard.allreduce_checksum(int(cs_out.item()), device=dev)
+    local_cs = int(cs_out.item()) & shard.MASK64
+    checksum = shard.allreduce_checksum(local_cs, device=coll_dev)
 
-    # e2e: host keys (pinned) -> rekey through the C ABI -> CHECKSUM -> 8 B back to host
+    # e2e through the public API: host keys (pinned) -> bsrng_rekey (staged
+    # H2D inside the call) -> bsrng_generate_host(CHECKSUM): the keystream
+    # kernel plus the 8 B device->host read of the result, stream-synchronised
     e2e = None
     if not args.no_e2e:
-        cs_host = torch.zeros(1, dtype=torch.int64).pin_memory()
+        cs_host = np.zeros(1, dtype=np.uint64)
+        kh, vh = keys_pin.numpy(), ivs_pin.numpy()
 
         def step_e2e(ev=None):
             if ev:
                 ev[2].record(stream)
-            g.rekey(keys_pin.numpy(), ivs_pin.numpy(), stream=stream)
+            g.rekey(kh, vh, stream=stream)
             if ev:
                 ev[0].record(stream)
-            g.generate(cs_out, bits, "checksum", stream=stream)
+            cs_host[:] = g.generate_host(bits, "checksum", stream=stream)
             if ev:
                 ev[1].record(stream)
-            with torch.cuda.stream(stream):
-                cs_host.copy_(cs_out, non_blocking=True)
 
         ms_e2e, _, _, _ = timed(step_e2e, max(1, args.steps), 1)
         e2e = {"value": n_total * bits / (ms_e2e * 1e-3) / 1e12, "unit": "Tb/s",
                "h2d_bytes_per_step": int(keys_h.nbytes + ivs_h.nbytes), "d2h_bytes_per_step": 8,
-               "ms_per_step": ms_e2e, "mode": "consume"}
+               "ms_per_step": ms_e2e, "mode": "consume",
+               "api": "bsrng_rekey(host keys/IVs) + bsrng_generate_host(CHECKSUM)",
+               "checksum_matches_device_path": bool(int(cs_host[0]) == local_cs)}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(cipher=args.cipher)
     context = None
     if rank == 0 and world == 1 and not args.no_context:
-        context = run_context(local_rank)
+        context = dict(peak_ctx, **run_context(dev.index, ("curand", "write_peak")))
 
     if rank == 0:
         head = results[args.mode]
@@ -540,12 +586,14 @@ def run_ours(args, rank, world, local_rank):
             "config": {"workload": f"{desc} ({args.mode})", "instances_total": n_total,
                        "instances_per_gpu": n, "bits_per_instance": bits,
                        "mode": args.mode, "parallelism": f"instance-range shards x{world}",
+                       "backend": args.backend if world > 1 else None,
                        "l2": (f"flushed (256 MiB write) between timed steps; state "
                               f"{state_words(args.cipher) * (n // 32) * 4 / 2**20:.0f} MiB, keys/IVs "
                               f"{n * key_iv_bytes(args.cipher) / 2**20:.0f} MiB")},
             "roofline": rf, "clocks": head.get("clocks"), "gpu_launches": head["gpu_launches"],
             "e2e": e2e, "cpu_baseline": cpu, "checksum": f"{checksum:016x}", "context": context,
             "modes": {m: {k: v for k, v in r.items() if k != "clocks"} for m, r in results.items()},
+            "clocks_by_mode": {m: r.get("clocks") for m, r in results.items()},
             "paper_context": "2.72 Tb/s RTX 2080 Ti, 2.90 Tb/s V100 (PAPER.md:46-50, 852-854); "
                              "exceeds the bit-exact LOP3 bound on those GPUs, see BASELINE.md",
         }
@@ -566,8 +614,12 @@ def main():
     if world > 1:
         import torch
         import torch.distributed as dist
-        torch.cuda.set_device(local_rank)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        dev = torch.device("cuda", local_rank % max(1, torch.cuda.device_count()))
+        torch.cuda.set_device(dev)
+        if args.backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
     try:
         run_ours(args, rank, world, local_rank)
     finally:
