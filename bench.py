@@ -40,7 +40,9 @@ BITS_DEFAULT = 1 << 20
 #    numerator the contract fixes: MICKEY 2.0 327 per clock (the spec's Galois
 #    form, output op included), Grain v1 39 (App. D's
 #    decomposition), AES-128-CTR 17280 per 32-block encryption (4096 bit
-#    positions; DESIGN.md sec. 5 AES), the LFSR's Eq. 2 feedback 2 (k = 4 taps).
+#    positions; DESIGN.md sec. 5 AES), the LFSR's Eq. 2 feedback 2 (k = 4 taps;
+#    + 1 to accumulate the output word in consume mode, as MICKEY's 327
+#    counts its output op).
 #  * KERNEL -- what the shipped kernels need: MICKEY 304 with the R reduction
 #    deferred over K = 4-clock blocks (315.5 at K = 2; mickey2.cuh clock_lazy,
 #    DESIGN.md sec. 5 item 10), Grain 37 (+1 to fold into the checksum), AES
@@ -49,6 +51,11 @@ BITS_DEFAULT = 1 << 20
 MICKEY2_GALOIS_OPS = 327.0
 MICKEY2_OPS_BY_BLOCK = {1: 327.0, 2: 315.5, 4: 304.0}
 ALGORITHMIC_OPS = {"mickey2": 327.0, "grain": 39.0, "aes128ctr": 17280.0 / 128.0, "lfsr128": 2.0}
+
+
+def algorithmic_ops(cipher, mode):
+    """SURVEY.md sec. 8(d) per-clock LOP3 count per 32-instance group."""
+    return 3.0 if (cipher == "lfsr128" and mode == "consume") else ALGORITHMIC_OPS[cipher]
 
 
 def mickey2_block(unroll):
@@ -117,7 +124,10 @@ def parse():
 
 # ------------------------------------------------------------------ helpers
 class ClockSampler:
-    """nvidia-smi clocks/throttle sampling during the timed region."""
+    """nvidia-smi clocks/throttle sampling (every 50 ms) during the timed
+    region: the sampler starts before the warm-up, waits for its first sample
+    (nvidia-smi takes ~0.1-0.5 s to start), and only samples that arrive
+    between begin() and end() (host clock) are reported."""
     Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
          "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
          "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
@@ -125,7 +135,8 @@ class ClockSampler:
     def __init__(self, index):
         self.index = index
         self.proc = None
-        self.lines = []
+        self.lines = []  # (arrival time, line)
+        self.t0 = self.t1 = None
 
     def start(self):
         try:
@@ -134,16 +145,26 @@ class ClockSampler:
                  "-lms", "50"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
+            deadline = time.time() + 5.0
+            while not self.lines and time.time() < deadline and self.proc.poll() is None:
+                time.sleep(0.02)
         except FileNotFoundError:
             self.proc = None
 
     def _read(self):
         for line in self.proc.stdout:
-            self.lines.append(line.strip())
+            self.lines.append((time.time(), line.strip()))
+
+    def begin(self):
+        self.t0 = time.time()
+
+    def end(self):
+        self.t1 = time.time()
 
     def stop(self):
         if not self.proc:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.06)  # let the last in-window sample arrive
         self.proc.terminate()
         try:
             self.proc.wait(timeout=5)
@@ -151,7 +172,11 @@ class ClockSampler:
             self.proc.kill()
         sm, mx, reasons = [], [], set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for ln in self.lines:
+        t0 = self.t0 if self.t0 is not None else 0.0
+        t1 = (self.t1 if self.t1 is not None else time.time()) + 0.05
+        for ts, ln in self.lines:
+            if not (t0 <= ts <= t1):
+                continue
             f = [x.strip() for x in ln.split(",")]
             if len(f) < 9:
                 continue
@@ -165,7 +190,8 @@ class ClockSampler:
                     reasons.add(nm)
         return {"sm_mhz": float(np.median(sm)) if sm else None,
                 "sm_max_mhz": max(mx) if mx else None,
-                "reasons": sorted(reasons), "samples": len(sm)}
+                "reasons": sorted(reasons), "samples": len(sm),
+                "window_s": round(t1 - 0.05 - t0, 3) if self.t0 is not None else None}
 
 
 def measured_peaks():
@@ -430,13 +456,15 @@ def run_ours(args, rank, world, local_rank):
             ev[1].record(stream)
 
     def timed(step_fn, steps, warmup, sampler=None):
+        if sampler:
+            sampler.start()
         for _ in range(warmup):
             step_fn()
         torch.cuda.synchronize(dev)
         step_ms, kern_ms, rekey_ms = [], [], []
         l0 = bsrng.launch_count()
         if sampler:
-            sampler.start()
+            sampler.begin()
         for _ in range(steps):
             flush.zero_()  # L2 flush between timed steps (outside the timed region)
             torch.cuda.synchronize(dev)
@@ -452,6 +480,8 @@ def run_ours(args, rank, world, local_rank):
             step_ms.append(e0.elapsed_time(e1))
             kern_ms.append(k0.elapsed_time(k1))
             rekey_ms.append(r0.elapsed_time(k0))
+        if sampler:
+            sampler.end()
         clocks = sampler.stop() if sampler else None
         launches = bsrng.launch_count() - l0
         # MAX over ranks of each rank's summed step / kernel / rekey times
@@ -486,7 +516,7 @@ def run_ours(args, rank, world, local_rank):
         before the timed region); the derived 148 x 64 lanes x sm_max peak and
         the kernel's own op count are reported beside it."""
         unroll = dict(kv.split("=", 1) for kv in args.opt).get("unroll")
-        alg = ALGORITHMIC_OPS[args.cipher]
+        alg = algorithmic_ops(args.cipher, mode)
         kops = lop3_per_bit(args.cipher, mode, int(unroll) if unroll else None)
         units = (n // 32) * bits / (kern_ms_per_step * 1e-3) / 1e12  # group-clocks per s, x 1e12
         peak = measured_peak or derived_peak

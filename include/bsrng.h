@@ -190,8 +190,11 @@ int64_t bsrng_copy_state(const bsrng_t* h, uint32_t* host_out, uint64_t words);
  *   "ctas_per_sm": resident CTAs per SM for the persistent grid (0 = auto)
  *   "unroll"     : clocks per loop iteration: Grain / LFSR 32 (default) or 16;
  *                  MICKEY 4 (the only one built); 0 = default
- *   "rm_ws"      : ROW_MAJOR kernel: -1 auto, 1 warp-specialised (AES: block-
- *                  lane), 0 plain
+ *   "rm_ws"      : ROW_MAJOR kernel: -1 auto, 1 warp-specialised (a clock-loop
+ *                  warp and a writer warp per SMSP; the writer transposes into
+ *                  tensor memory and flushes 64 B per row; auto for the LFSR,
+ *                  and for Grain when every warp-unit gets its own SMSP; AES:
+ *                  the block-lane kernel), 0 plain
  *   "rm_tmem"    : ROW_MAJOR plain kernel: stage the row segments in tensor
  *                  memory (TMEM, 256 columns per CTA, two CTAs per SM) (1)
  *                  or in shared memory (0); -1 = cipher default (MICKEY /
@@ -203,6 +206,10 @@ int64_t bsrng_copy_state(const bsrng_t* h, uint32_t* host_out, uint64_t words);
  *                  double-buffered staging (512 columns), the previous sector
  *                  period flushed 4 rows per block (1, default) or a single
  *                  buffer (0)
+ *   "rm_wide"    : ROW_MAJOR plain kernel: 64 B TMEM staging per row with one
+ *                  clock-loop warp per SMSP (1) or not (0, default)
+ *   "rm_l2last"  : ROW_MAJOR 32 B flushes (TMA / 8 B stores) with an L2
+ *                  evict_last hint (1, default) or evict-first (0)
  *   "init_fused" : create/rekey: slicing fused into the initialisation kernel
  *                  (1, default) or the separate ballot slice (+ preclock)
  *                  kernels (0)

@@ -126,6 +126,10 @@ struct Grain {
     // ...with time segments (~8 per resident warp): a lone Grain warp keeps
     // the ALU only ~70% busy, so a whole-unit tail wave would run slow
     static constexpr bool RM_SEGMENTED = true;
+    // ...unless the call has at most one warp-unit per SMSP (the paper's launch
+    // shape): lone clock-loop warps then get a writer warp each (rowmajor_ws.cuh;
+    // C4 5.82 vs 5.07 Tb/s)
+    static constexpr int RM_WS = 1;
     uint32_t s[80], b[80];
 
     __device__ __forceinline__ void load(const uint32_t* st, uint64_t Gp, uint64_t g)

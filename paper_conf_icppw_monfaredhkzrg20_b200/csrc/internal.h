@@ -92,6 +92,12 @@ struct bsrng {
     int opt_rm_tma = 1;
     // TMEM-staged ROW_MAJOR with one CTA per SM: double-buffered staging (1) or not (0)
     int opt_rm_dbl = 1;
+    // ROW_MAJOR: 64 B TMEM staging per row, one clock-loop warp per SMSP (1)
+    int opt_rm_wide = 0;
+    // ROW_MAJOR 32 B flushes with an L2 evict_last hint (1, default: a row's
+    // next sector then finds its 128 B line resident; Grain C2 11.5 vs 10.5
+    // Tb/s) or evict-first (0)
+    int opt_rm_l2last = 1;
     // init: slicing fused into the init kernel (1) or the ballot slice kernels (0)
     int opt_init_fused = 1;
 };

@@ -132,6 +132,8 @@ struct KsArgs {
     // flushed 4 rows per block during the next period (lone clock-loop warps
     // cannot otherwise hide the flush)
     int tmem_dbl;
+    // ROW_MAJOR 32 B flushes (TMA / 8 B sector stores): L2 evict_last hint
+    int l2last;
     uint64_t tma_groups;
     CUtensorMap tmap;  // 3-D view of `out`: [q 32][group][byte], see bsrng.cu
 };
@@ -336,10 +338,10 @@ __device__ __forceinline__ void tmem_st1(uint32_t taddr, uint32_t v)
 {
     asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0+%2], {%1};" ::"r"(taddr), "r"(v), "n"(OFF) : "memory");
 }
-template <int H, int... Q>
+template <int H, int RS, int... Q>
 __device__ __forceinline__ void tmem_st_rows(uint32_t base, const uint32_t (&x)[16], std::integer_sequence<int, Q...>)
 {
-    (tmem_st1<(16 * H + Q) * 8>(base, x[Q]), ...);
+    (tmem_st1<(16 * H + Q) * RS>(base, x[Q]), ...);
 }
 
 // v[0..15] <- 16 consecutive columns of this thread's lane (load + wait in one
@@ -359,8 +361,10 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&v)[16])
 __device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 
 // Transpose 32 z words held in registers and park the row words of slot k in
-// TMEM columns q*8 + k (tm = this warp's lane-quarter base address).
-template <bool MSB_FIRST>
+// TMEM columns q*RS + k (tm = this warp's lane-quarter base address; RS = 8
+// slots per row, or 16 for the 64 B staging, where k is already the permuted
+// column wide_col(slot)).
+template <bool MSB_FIRST, int RS = 8>
 __device__ __forceinline__ void rowmajor_transpose_tmem(const uint32_t (&z)[32], uint32_t tm, uint32_t k)
 {
     constexpr int X = MSB_FIRST ? 7 : 0;
@@ -371,13 +375,13 @@ __device__ __forceinline__ void rowmajor_transpose_tmem(const uint32_t (&z)[32],
         for (int q = 0; q < 16; ++q) x[q] = __byte_perm(z[q ^ X], z[(q + 16) ^ X], h == 0 ? 0x5410 : 0x7632);
         bt_transpose16(x);
         if (h == 0)
-            tmem_st_rows<0>(tm + k, x, std::make_integer_sequence<int, 16>{});
+            tmem_st_rows<0, RS>(tm + k, x, std::make_integer_sequence<int, 16>{});
         else
-            tmem_st_rows<1>(tm + k, x, std::make_integer_sequence<int, 16>{});
+            tmem_st_rows<1, RS>(tm + k, x, std::make_integer_sequence<int, 16>{});
     }
 }
 // The same from 32 z words staged in shared memory ([t][lane], zs = lane's column).
-template <bool MSB_FIRST>
+template <bool MSB_FIRST, int RS = 8>
 __device__ __forceinline__ void rowmajor_transpose_smem_tmem(const uint32_t* zs, uint32_t tm, uint32_t k)
 {
     constexpr int X = MSB_FIRST ? 7 : 0;
@@ -389,9 +393,9 @@ __device__ __forceinline__ void rowmajor_transpose_smem_tmem(const uint32_t* zs,
             x[q] = __byte_perm(zs[(q ^ X) * 32], zs[((q + 16) ^ X) * 32], h == 0 ? 0x5410 : 0x7632);
         bt_transpose16(x);
         if (h == 0)
-            tmem_st_rows<0>(tm + k, x, std::make_integer_sequence<int, 16>{});
+            tmem_st_rows<0, RS>(tm + k, x, std::make_integer_sequence<int, 16>{});
         else
-            tmem_st_rows<1>(tm + k, x, std::make_integer_sequence<int, 16>{});
+            tmem_st_rows<1, RS>(tm + k, x, std::make_integer_sequence<int, 16>{});
     }
 }
 
@@ -453,6 +457,32 @@ __device__ __forceinline__ uint8_t* add_fma(uint8_t* p, uint64_t d)
     return reinterpret_cast<uint8_t*>(r);
 }
 
+__device__ __forceinline__ uint64_t l2_evict_last_policy()
+{
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ void st128_hint(uint8_t* p, uint32_t a, uint32_t b, uint32_t c, uint32_t d, uint64_t pol)
+{
+    asm volatile("st.global.L2::cache_hint.v4.u32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(p), "r"(a), "r"(b), "r"(c),
+                 "r"(d), "l"(pol)
+                 : "memory");
+}
+__device__ __forceinline__ void st64_hint(uint8_t* p, uint32_t a, uint32_t b, uint64_t pol)
+{
+    asm volatile("st.global.L2::cache_hint.v2.u32 [%0], {%1, %2}, %3;" ::"l"(p), "r"(a), "r"(b), "l"(pol) : "memory");
+}
+// 8 B sector-flush store: evict-first (streaming), or with an L2 evict_last
+// hint (pol != 0) so a row's next sector finds its 128 B line still resident
+__device__ __forceinline__ void st_sector8(uint8_t* p, uint32_t a, uint32_t b, uint64_t pol)
+{
+    if (pol)
+        st64_hint(p, a, b, pol);
+    else
+        __stcs(reinterpret_cast<uint2*>(p), make_uint2(a, b));
+}
+
 // v[0..15] <- tcgen05.ld.16x256b.x4 at taddr: thread t receives, for repeat
 // i = 0..3 (columns +8i), TMEM lane base+t/4 columns 2(t%4), 2(t%4)+1 in
 // v[4i], v[4i+1] and lane base+8+t/4 (same columns) in v[4i+2], v[4i+3]
@@ -478,9 +508,11 @@ __device__ __forceinline__ void tmem_ld16x256b_x4(uint32_t taddr, uint32_t (&v)[
 // samples).  row0s / nvalids: this warp's per-thread row bases and row counts
 // (shared memory, indexed by the thread = TMEM lane that computed them).
 __device__ __forceinline__ void rowmajor_store_tmem_sectors(uint32_t tm, uint8_t* const* row0s,
-                                                            const uint32_t* nvalids, uint64_t row_bytes, uint64_t col)
+                                                            const uint32_t* nvalids, uint64_t row_bytes, uint64_t col,
+                                                            bool l2last = false)
 {
     tmem_wait_st();
+    const uint64_t pol = l2last ? l2_evict_last_policy() : 0ull;
     const uint32_t t = laneid_volatile();
 #pragma unroll 1
     for (uint32_t h = 0; h < 2; ++h) {
@@ -499,8 +531,8 @@ __device__ __forceinline__ void rowmajor_store_tmem_sectors(uint32_t tm, uint8_t
                 tmem_ld16x256b_x4(tm + ((16 * h) << 16) + q0 * 8, v);
 #pragma unroll
                 for (int i = 0; i < 4; ++i) {
-                    __stcs(reinterpret_cast<uint2*>(pa), make_uint2(v[4 * i], v[4 * i + 1]));
-                    __stcs(reinterpret_cast<uint2*>(pb), make_uint2(v[4 * i + 2], v[4 * i + 3]));
+                    st_sector8(pa, v[4 * i], v[4 * i + 1], pol);
+                    st_sector8(pb, v[4 * i + 2], v[4 * i + 3], pol);
                     pa = add_fma(pa, row_bytes);
                     pb = add_fma(pb, row_bytes);
                 }
@@ -541,9 +573,10 @@ __device__ __forceinline__ void rowmajor_store_tmem_sectors(uint32_t tm, uint8_t
 // row real and 8 B aligned (tmem_dbl's progressive flush): 16x256b read-back,
 // unpredicated 8 B stores.
 __device__ __forceinline__ void rowmajor_store_tmem_rows(uint32_t tm, uint8_t* const* row0s, uint64_t row_bytes,
-                                                         uint64_t col, uint32_t q_lo, uint32_t q_hi)
+                                                         uint64_t col, uint32_t q_lo, uint32_t q_hi, bool l2last = false)
 {
     tmem_wait_st();
+    const uint64_t pol = l2last ? l2_evict_last_policy() : 0ull;
     const uint32_t t = laneid_volatile();
 #pragma unroll 1
     for (uint32_t h = 0; h < 2; ++h) {
@@ -556,11 +589,110 @@ __device__ __forceinline__ void rowmajor_store_tmem_rows(uint32_t tm, uint8_t* c
             tmem_ld16x256b_x4(tm + ((16 * h) << 16) + q0 * 8, v);
 #pragma unroll
             for (int i = 0; i < 4; ++i) {
-                __stcs(reinterpret_cast<uint2*>(pa), make_uint2(v[4 * i], v[4 * i + 1]));
-                __stcs(reinterpret_cast<uint2*>(pb), make_uint2(v[4 * i + 2], v[4 * i + 3]));
+                st_sector8(pa, v[4 * i], v[4 * i + 1], pol);
+                st_sector8(pb, v[4 * i + 2], v[4 * i + 3], pol);
                 pa += row_bytes;
                 pb += row_bytes;
             }
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// 64 B staging ("wide": one clock-loop warp per SMSP owns all 512 TMEM
+// columns of its lane quarter).  Row q's 16 slot words live at columns
+// q*16 + wide_col(k), permuted so that the tcgen05.ld.16x256b read-back hands
+// thread j = t%4 the slots 4j..4j+3 -- 16 contiguous bytes -- of the rows in
+// TMEM lanes t/4 and t/4+8: every STG.128 writes 8 rows x 64 B.  Why 64 B:
+// the flush_pattern microbenchmark (profiles/r2_flush_pattern.log) writes the
+// kernels' output pattern (1024 rows per warp, one piece per row per flush)
+// without compute: 32 B per row per flush reaches 1.4-1.8 TB/s, 64 B 2.9-3.6
+// TB/s (DRAM page locality).  The stores carry an L2 evict_last hint (3.55 vs
+// 2.93 TB/s at 64 B): a row's next piece lands on the same 128 B line.
+// ---------------------------------------------------------------------------
+__host__ __device__ constexpr uint32_t wide_col(uint32_t k)
+{
+    return 2 * (k >> 2) + (k & 1) + ((k & 2) ? 8 : 0);
+}
+
+
+// Whole 64 B flush (slots 0..15 of every row; rows 8 B aligned: 16 B
+// aligned rows take one STG.128 per row piece, 8 B aligned ones -- e.g. the
+// paper shape's 552 B rows -- two STG.64).  row0s / nvalids: this warp's
+// per-thread row bases and real-row counts (smem).
+__device__ __forceinline__ void st_piece16(uint8_t* p, uint32_t a, uint32_t b, uint32_t c, uint32_t d, uint64_t pol,
+                                           bool a16)
+{
+    if (a16) {
+        st128_hint(p, a, b, c, d, pol);
+    } else {
+        st64_hint(p, a, b, pol);
+        st64_hint(p + 8, c, d, pol);
+    }
+}
+__device__ __forceinline__ void rowmajor_store_tmem_wide(uint32_t tm, uint8_t* const* row0s, const uint32_t* nvalids,
+                                                         uint64_t row_bytes, uint64_t col)
+{
+    tmem_wait_st();
+    const uint32_t t = laneid_volatile();
+    const uint64_t pol = l2_evict_last_policy();
+    const bool a16 = ((row_bytes | col) & 15) == 0;
+#pragma unroll 1
+    for (uint32_t h = 0; h < 2; ++h) {
+        const uint32_t la = 16 * h + (t >> 2), lb = la + 8;
+        uint8_t* pa = row0s[la] + col + 16 * (t & 3);
+        uint8_t* pb = row0s[lb] + col + 16 * (t & 3);
+        const uint32_t na = nvalids[la], nb = nvalids[lb];
+        if (a16 && __all_sync(0xFFFFFFFFu, (na & nb) == 32)) {
+#pragma unroll 1
+            for (uint32_t q = 0; q < 32; q += 2) {
+                uint32_t v[16];  // rows q (v0..7) and q+1 (v8..15) of lanes la (v[4i], v[4i+1]) / lb
+                tmem_ld16x256b_x4(tm + ((16 * h) << 16) + q * 16, v);
+                st128_hint(pa, v[0], v[1], v[4], v[5], pol);
+                st128_hint(pb, v[2], v[3], v[6], v[7], pol);
+                pa = add_fma(pa, row_bytes);
+                pb = add_fma(pb, row_bytes);
+                st128_hint(pa, v[8], v[9], v[12], v[13], pol);
+                st128_hint(pb, v[10], v[11], v[14], v[15], pol);
+                pa = add_fma(pa, row_bytes);
+                pb = add_fma(pb, row_bytes);
+            }
+            continue;
+        }
+#pragma unroll 1
+        for (uint32_t q = 0; q < 32; q += 2) {
+            uint32_t v[16];
+            tmem_ld16x256b_x4(tm + ((16 * h) << 16) + q * 16, v);
+            if (q < na) st_piece16(pa, v[0], v[1], v[4], v[5], pol, a16);
+            if (q < nb) st_piece16(pb, v[2], v[3], v[6], v[7], pol, a16);
+            pa += row_bytes;
+            pb += row_bytes;
+            if (q + 1 < na) st_piece16(pa, v[8], v[9], v[12], v[13], pol, a16);
+            if (q + 1 < nb) st_piece16(pb, v[10], v[11], v[14], v[15], pol, a16);
+            pa += row_bytes;
+            pb += row_bytes;
+        }
+    }
+}
+
+// Partial 64 B flush: slots [k_lo, k_hi] of this thread's own rows, word by
+// word (item boundaries that are not whole 512-clock periods, rows that are
+// not 16 B aligned).  The 32x32b loads are warp-collective: every lane runs them.
+__device__ __forceinline__ void rowmajor_store_tmem_wide_partial(uint32_t tm, uint8_t* row0, uint64_t row_bytes,
+                                                                 uint32_t nvalid, uint32_t k_lo, uint32_t k_hi,
+                                                                 uint64_t col)
+{
+    tmem_wait_st();
+    uint8_t* p = row0 + col;
+#pragma unroll 1
+    for (uint32_t q = 0; q < 32; ++q) {
+        uint32_t v[16];  // v[wide_col(k)] = slot k of row q
+        tmem_ld16(tm + q * 16, v);
+        if (q < nvalid) {
+#pragma unroll
+            for (int k = 0; k < 16; ++k)
+                if (uint32_t(k) >= k_lo && uint32_t(k) <= k_hi)
+                    __stcs(reinterpret_cast<uint32_t*>(p + q * row_bytes) + (k - k_lo), v[wide_col(k)]);
         }
     }
 }
@@ -571,6 +703,15 @@ __device__ __forceinline__ uint32_t smem_addr_u32(const void* p)
 }
 __device__ __forceinline__ void bulk_wait_read_all() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void tma_store_3d_hint(const CUtensorMap* map, uint32_t src, int c0, int c1, int c2,
+                                                  uint64_t pol)
+{
+    asm volatile(
+        "cp.async.bulk.tensor.3d.global.shared::cta.bulk_group.L2::cache_hint [%0, {%2, %3, %4}], [%1], %5;" ::"l"(
+            reinterpret_cast<uint64_t>(map)),
+        "r"(src), "r"(c0), "r"(c1), "r"(c2), "l"(pol)
+        : "memory");
+}
 __device__ __forceinline__ void tma_store_3d(const CUtensorMap* map, uint32_t src, int c0, int c1, int c2)
 {
     asm volatile("cp.async.bulk.tensor.3d.global.shared::cta.bulk_group [%0, {%2, %3, %4}], [%1];" ::"l"(
@@ -588,7 +729,7 @@ constexpr int TMA_BUF_WORDS = 4096;  // 16 KB per warp: two 8 KB boxes
 // right away cost 8.6% of Grain's ROW_MAJOR time (ncu: BSYNC after lane 0's
 // cp.async.bulk.wait_group.read).
 __device__ __forceinline__ void tma_flush_half(uint32_t tm, uint32_t* buf, const CUtensorMap* map, uint64_t g_w0,
-                                               uint64_t col, uint32_t h)
+                                               uint64_t col, uint32_t h, bool l2last = false)
 {
     const uint32_t t = laneid_volatile();
     const uint32_t sb = smem_addr_u32(buf);
@@ -611,8 +752,14 @@ __device__ __forceinline__ void tma_flush_half(uint32_t tm, uint32_t* buf, const
     __syncwarp();
     if (t == 0) {
         const int g = int(g_w0 + 16 * h);
-        tma_store_3d(map, sb, int(col), g, 0);
-        tma_store_3d(map, sb + 8192, int(col), g + 8, 0);
+        if (l2last) {
+            const uint64_t pol = l2_evict_last_policy();
+            tma_store_3d_hint(map, sb, int(col), g, 0, pol);
+            tma_store_3d_hint(map, sb + 8192, int(col), g + 8, 0, pol);
+        } else {
+            tma_store_3d(map, sb, int(col), g, 0);
+            tma_store_3d(map, sb + 8192, int(col), g + 8, 0);
+        }
         asm volatile("cp.async.bulk.commit_group;" ::: "memory");
     }
 }
@@ -629,7 +776,9 @@ __device__ __forceinline__ void next_item(const KsArgs& a, volatile uint32_t* sl
 // memory instead (8 slots, no smem for rows); ZREG: see rm_warp_words.
 // DBL: double-buffered TMEM staging (KsArgs::tmem_dbl), a separate instance so
 // the single-buffer kernel carries none of its code (measured: 0.3%)
-template <class C, int LAYOUT, int U, int BLOCK, int SLOTS = 8, bool ZREG = true, bool TMEM = false, bool DBL = false>
+// WIDE: 64 B TMEM staging per row (one CTA per SM, all 512 columns, 16 slots).
+template <class C, int LAYOUT, int U, int BLOCK, int SLOTS = 8, bool ZREG = true, bool TMEM = false, bool DBL = false,
+          bool WIDE = false>
 __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant__ KsArgs a)
 {
     static_assert(32 % U == 0, "U must divide 32");
@@ -659,7 +808,8 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
     __shared__ uint32_t s_tmem;
     if constexpr (LAYOUT == L_ROW_MAJOR && TMEM) {
         static_assert(BLOCK == 128, "TMEM staging maps warp w to lane quarter w");
-        (void)tmem_alloc_cta(&s_tmem, DBL);
+        static_assert(!(DBL && WIDE), "one 512-column TMEM use at a time");
+        (void)tmem_alloc_cta(&s_tmem, DBL || WIDE);
         if (laneid_volatile() == 0) s_pend_col[threadIdx.x >> 5] = s_pdbl_col[threadIdx.x >> 5] = 0;
     }
     // tmem_dbl: sector period B >> 3 stages into buffer (B >> 3) & 1
@@ -677,7 +827,7 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
             const uint64_t pc = *reinterpret_cast<volatile uint64_t*>(&s_pend_col[wq]);
             if (pc) {
                 tma_flush_half(tm_addr(), tma_buf(), &a.tmap, *reinterpret_cast<volatile uint64_t*>(&s_pend_g[wq]),
-                               pc - 1, 1);
+                               pc - 1, 1, a.l2last);
                 __syncwarp();
                 if (laneid_volatile() == 0) s_pend_col[wq] = 0;
                 __syncwarp();
@@ -780,7 +930,10 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
                 s_nblk[threadIdx.x >> 5] = uint32_t(nclk >> 5);
             }
             __syncwarp();
-            constexpr uint32_t NSLOT = TMEM ? 8 : SLOTS;
+            constexpr uint32_t NSLOT = TMEM ? (WIDE ? 16 : 8) : SLOTS;
+            constexpr int RS = WIDE ? 16 : 8;  // TMEM columns per row
+            // TMEM column of slot k (WIDE: permuted for the 16x256b read-back)
+            auto tcol = [&](uint64_t B, uint32_t k) { return WIDE ? wide_col(k) : dbl_off(B) + k; };
             constexpr int WW = TMEM ? ZS_WORDS : rm_warp_words(U, SLOTS, ZREG);
             // re-derived after every clock loop from non-CSE-able special registers
             auto zs_ptr = [&]() { return rm_smem + (tid_volatile() >> 5) * WW + laneid_volatile(); };
@@ -802,7 +955,7 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
                     const uint32_t k = uint32_t(B & (NSLOT - 1));
                     tma_pending();
                     if constexpr (TMEM)
-                        rowmajor_transpose_tmem<C::MSB_FIRST>(zr, tm_addr() + dbl_off(B), k);
+                        rowmajor_transpose_tmem<C::MSB_FIRST, RS>(zr, tm_addr(), tcol(B, k));
                     else
                         rowmajor_transpose_regs<C::MSB_FIRST, SLOTS>(zr, os_ptr(), k);
                 } else {
@@ -819,7 +972,7 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
                     const uint32_t k = uint32_t(B & (NSLOT - 1));
                     tma_pending();
                     if constexpr (TMEM)
-                        rowmajor_transpose_smem_tmem<C::MSB_FIRST>(zs_ptr(), tm_addr() + dbl_off(B), k);
+                        rowmajor_transpose_smem_tmem<C::MSB_FIRST, RS>(zs_ptr(), tm_addr(), tcol(B, k));
                     else
                         rowmajor_transpose<C::MSB_FIRST, SLOTS>(zs_ptr(), os_ptr(), k);
                 }
@@ -834,7 +987,7 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
                         if (pc) {
                             const uint32_t q_hi = blk + 1 == nblk ? 32u : 4 * k + 4;
                             rowmajor_store_tmem_rows(tm_addr() + (dbl_off(B) ^ TMEM_COLS), s_row0 + wq * 32,
-                                                     a.row_bytes, pc - 1, 4 * k, q_hi);
+                                                     a.row_bytes, pc - 1, 4 * k, q_hi, a.l2last);
                             if (q_hi == 32) {
                                 __syncwarp();
                                 if (laneid_volatile() == 0) s_pdbl_col[wq] = 0;
@@ -850,7 +1003,17 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
                     if constexpr (TMEM) {
                         const uint64_t g_w0 = (*slot % a.units) * 32u;  // the warp's first group
                         const bool full_real = __all_sync(0xFFFFFFFFu, s_nvalid[t] == 32);
-                        if (DBL && k_lo == 0 && k == 7 && blk + 1 < nblk && full_real &&
+                        if constexpr (WIDE) {
+                            (void)full_real;
+                            (void)g_w0;
+                            if (k_lo == 0 && k == NSLOT - 1 && ((a.row_bytes | col) & 7) == 0 &&
+                                a.row_bytes < (1ull << 32))
+                                rowmajor_store_tmem_wide(tm_addr(), s_row0 + (t & ~31u), s_nvalid + (t & ~31u),
+                                                         a.row_bytes, col);
+                            else
+                                rowmajor_store_tmem_wide_partial(tm_addr(), s_row0[t], a.row_bytes, s_nvalid[t],
+                                                                 k_lo, k, col);
+                        } else if (DBL && k_lo == 0 && k == 7 && blk + 1 < nblk && full_real &&
                             ((a.row_bytes | col) & 7) == 0) {
                             // flushed during the next period (other buffer)
                             __syncwarp();
@@ -858,7 +1021,7 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
                             __syncwarp();
                         } else if (a.use_tma && k_lo == 0 && k == 7 && g_w0 + 32 <= a.tma_groups) {
                             tmem_wait_st();
-                            tma_flush_half(tm_addr(), tma_buf(), &a.tmap, g_w0, col, 0);
+                            tma_flush_half(tm_addr(), tma_buf(), &a.tmap, g_w0, col, 0, a.l2last);
                             if (blk + 1 < nblk) {  // defer the second half to the next block
                                 if (laneid_volatile() == 0) {
                                     s_pend_col[t >> 5] = col + 1;
@@ -866,11 +1029,11 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
                                 }
                                 __syncwarp();
                             } else {
-                                tma_flush_half(tm_addr(), tma_buf(), &a.tmap, g_w0, col, 1);
+                                tma_flush_half(tm_addr(), tma_buf(), &a.tmap, g_w0, col, 1, a.l2last);
                             }
                         } else if (k_lo == 0 && k == 7 && ((a.row_bytes | col) & 7) == 0 && a.row_bytes < (1ull << 32))
                             rowmajor_store_tmem_sectors(tm_addr() + dbl_off(B), s_row0 + (t & ~31u),
-                                                        s_nvalid + (t & ~31u), a.row_bytes, col);
+                                                        s_nvalid + (t & ~31u), a.row_bytes, col, a.l2last);
                         else
                             rowmajor_store_tmem(tm_addr() + dbl_off(B), s_row0[t], a.row_bytes, s_nvalid[t], k_lo, k,
                                                 col);
@@ -914,7 +1077,7 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
     if constexpr (LAYOUT == L_ROW_MAJOR && TMEM) {
         if (a.use_tma && laneid_volatile() == 0) bulk_wait_all();  // smem boxes read, stores done
         __syncwarp();
-        tmem_dealloc_cta(*reinterpret_cast<volatile uint32_t*>(&s_tmem), DBL);
+        tmem_dealloc_cta(*reinterpret_cast<volatile uint32_t*>(&s_tmem), DBL || WIDE);
     }
 }
 

@@ -7,7 +7,8 @@
 //   ROW_MAJOR, smem       : keystream_kernel<C, ROW_MAJOR, U>         (8 sector slots, z block in regs at U = 32)
 //   ROW_MAJOR, TMEM       : keystream_kernel<C, ROW_MAJOR, U, .., TMEM>
 //   ROW_MAJOR, TMEM + dbl : keystream_kernel<C, ROW_MAJOR, U, .., TMEM, DBL>
-//   ROW_MAJOR, specialised: keystream_rm_ws_kernel<C, U>
+//   ROW_MAJOR, TMEM 64 B  : keystream_kernel<C, ROW_MAJOR, U, .., TMEM, -, WIDE>
+//   ROW_MAJOR, specialised: keystream_rm_ws_kernel<C, U>   (compute + writer warps, TMEM 64 B staging)
 #pragma once
 #include <algorithm>
 #include <cstdio>
@@ -21,15 +22,15 @@ namespace bsrng_impl {
 
 constexpr int KS_BLOCK = 128;
 
-template <class C, int LAYOUT, bool TMEM = false, bool DBL = false>
+template <class C, int LAYOUT, bool TMEM = false, bool DBL = false, bool WIDE = false>
 auto pick_keystream_kernel(const bsrng_t* h, int* U)
 {
-    auto kern = &bsk::keystream_kernel<C, LAYOUT, C::U_DEFAULT, KS_BLOCK, 8, true, TMEM, DBL>;
+    auto kern = &bsk::keystream_kernel<C, LAYOUT, C::U_DEFAULT, KS_BLOCK, 8, true, TMEM, DBL, WIDE>;
     *U = C::U_DEFAULT;
     if (h->opt_unroll == C::U_ALT0)
-        kern = &bsk::keystream_kernel<C, LAYOUT, C::U_ALT0, KS_BLOCK, 8, true, TMEM, DBL>, *U = C::U_ALT0;
+        kern = &bsk::keystream_kernel<C, LAYOUT, C::U_ALT0, KS_BLOCK, 8, true, TMEM, DBL, WIDE>, *U = C::U_ALT0;
     if (h->opt_unroll == C::U_ALT1)
-        kern = &bsk::keystream_kernel<C, LAYOUT, C::U_ALT1, KS_BLOCK, 8, true, TMEM, DBL>, *U = C::U_ALT1;
+        kern = &bsk::keystream_kernel<C, LAYOUT, C::U_ALT1, KS_BLOCK, 8, true, TMEM, DBL, WIDE>, *U = C::U_ALT1;
     return kern;
 }
 
@@ -41,13 +42,21 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
     // 8 warps per CTA of which 4 run the clock loop; always persistent), or
     // the plain clock kernel with the row segments staged in tensor memory
     // (TMEM) or shared memory.  Defaults per cipher (RM_TMEM traits).
-    const bool ws_pref = h->opt_rm_ws < 0 ? (C::U_DEFAULT != 32 && !C::RM_TMEM) : (h->opt_rm_ws != 0);
+    // auto (C::RM_WS): 0 never, 1 when every warp-unit gets its own SMSP
+    // (lone clock-loop warps), 2 always
+    const bool lone = h->units <= uint64_t(h->num_sms) * 4;
+    const bool ws_pref = h->opt_rm_ws < 0 ? (C::RM_WS == 2 || (C::RM_WS == 1 && lone)) : (h->opt_rm_ws != 0);
     // calls longer than MAX_SEG_CLOCKS need time segments, i.e. the persistent queue
     const bool persistent = h->opt_sched != 0 || bits > MAX_SEG_CLOCKS;
     const bool ws = RM && ws_pref && persistent;
-    const bool tmem = RM && !ws && (h->opt_rm_tmem < 0 ? C::RM_TMEM : h->opt_rm_tmem > 0);
+    // 64 B TMEM staging (keystream.cuh wide_col): one clock-loop warp per
+    // SMSP with all 512 columns, so each flush writes 64 B per row
+    const bool wide = RM && !ws && h->opt_rm_wide > 0;
+    const bool tmem = wide || (RM && !ws && (h->opt_rm_tmem < 0 ? C::RM_TMEM : h->opt_rm_tmem > 0));
     int U = 0;
-    auto kern = tmem ? pick_keystream_kernel<C, LAYOUT, RM>(h, &U) : pick_keystream_kernel<C, LAYOUT>(h, &U);
+    auto kern = wide   ? pick_keystream_kernel<C, LAYOUT, RM, false, RM>(h, &U)
+                : tmem ? pick_keystream_kernel<C, LAYOUT, RM>(h, &U)
+                       : pick_keystream_kernel<C, LAYOUT>(h, &U);
     bsk::KsArgs a{};
     a.state = h->state;
     a.Gp = h->Gp;
@@ -62,13 +71,14 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
     a.row_bytes = bits / 8;
     a.units = h->units;
     a.scratch = h->sched + 1 + h->units;
+    a.l2last = h->opt_rm_l2last;
 
     int block = KS_BLOCK, compute_warps = KS_BLOCK / 32;
     size_t smem = RM ? size_t(KS_BLOCK / 32) * bsk::rm_warp_words(U, 8, true) * 4 : 0;
     if (tmem) smem = U == 32 ? 0 : size_t(KS_BLOCK / 32) * bsk::ZS_WORDS * 4;
     // TMA tensor stores for the whole-sector flushes of all-real warps: needs
     // 16 B aligned row strides (TMA global strides) and at least one such warp
-    if (tmem && h->opt_rm_tma && (a.row_bytes % 16) == 0 && h->n / 32 >= 32 && a.row_bytes < (1ull << 32)) {
+    if (tmem && !wide && h->opt_rm_tma && (a.row_bytes % 16) == 0 && h->n / 32 >= 32 && a.row_bytes < (1ull << 32)) {
         if (int rc = encode_rowmajor_tmap(&a.tmap, out, a.row_bytes, h->n / 32)) return rc;
         a.use_tma = 1;
         a.tma_groups = h->n / 32;
@@ -98,7 +108,7 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
         // The occupancy API reports 1 CTA/SM for kernels that allocate tensor
         // memory; registers (255 x 128 threads -> 2 CTAs) and TMEM (2 x 256 of
         // 512 columns) allow two, which the GPU then runs (ncu: 7.9 warps/SM).
-        if (tmem) occ_max = 2;
+        if (tmem) occ_max = wide ? 1 : 2;
         // Auto policy (opt_ctas_per_sm == 0).  Many more warp-units than warp
         // slots: two warps per SMSP, one item per unit (no time segments, so no
         // warp ever waits on another; a warp left alone at the end runs at
@@ -111,6 +121,7 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
             whole_units = !ws && occ_max >= 2 && h->units >= 3 * slots2 && !(tmem && C::RM_SEGMENTED);
             occ = (whole_units || tmem) ? 2 : 1;
         }
+        if (wide) occ = 1;
         // an explicit setting is honoured even above the occupancy API's
         // estimate (extra CTAs queue; the ticket order cannot deadlock)
         if (occ > occ_max && h->opt_ctas_per_sm <= 0) occ = occ_max;
@@ -124,13 +135,15 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
             // >= ~32 items per resident warp so the tail is <~3% of the call,
             // but segments no shorter than 256 clocks (state carry stays <1%)
             // (TMEM-staged ROW_MAJOR at two warps per SMSP: ~8 items per warp)
-            const uint64_t per_warp = tmem ? 8 : 32;
+            const uint64_t per_warp = (tmem && !wide) ? 8 : 32;
             nseg = std::max<uint64_t>(1, (per_warp * slots + h->units - 1) / h->units);
             nseg = std::min<uint64_t>(nseg, std::max<uint64_t>(1, bits / 256));
         }
         nseg = std::max<uint64_t>(nseg, (bits + MAX_SEG_CLOCKS - 1) / MAX_SEG_CLOCKS);
-        // whole 256-clock blocks keep ROW_MAJOR sector flushes full (32 B/row)
-        const uint64_t quantum = bits >= 256 ? 256 : 32;
+        // whole 256-clock blocks keep ROW_MAJOR sector flushes full (32 B/row;
+        // 512 clocks = 64 B for the wide staging)
+        const uint64_t q_full = (wide || ws) ? 512 : 256;
+        const uint64_t quantum = bits >= q_full ? q_full : 32;
         uint64_t seg = ((bits + nseg - 1) / nseg + quantum - 1) / quantum * quantum;
         nseg = (bits + seg - 1) / seg;
         a.persistent = 1;
@@ -148,7 +161,7 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
     // second CTA queued behind a 512-column allocation cannot deadlock): the
     // lone clock-loop warps get double-buffered TMEM staging (KsArgs::tmem_dbl)
     if constexpr (RM) {
-        if (tmem && !a.use_tma && h->opt_rm_dbl && a.nseg == 1 && grid <= unsigned(h->num_sms)) {
+        if (tmem && !wide && !a.use_tma && h->opt_rm_dbl && a.nseg == 1 && grid <= unsigned(h->num_sms)) {
             a.tmem_dbl = 1;
             kern = pick_keystream_kernel<C, LAYOUT, true, true>(h, &U);
             if (int rc = set_smem(reinterpret_cast<const void*>(kern), smem)) return rc;

@@ -6,16 +6,22 @@
 //
 //   compute warp c (wid 0..3, one per SMSP): runs the register-resident clock
 //     loop of the time-segmented persistent queue (keystream.cuh) and writes
-//     one slice word per clock into a double-buffered z block in smem;
-//   writer warp c+4 (same SMSP): for every 32-clock block transposes each
-//     thread's 32x32 bit tile (PRMT + IMAD-shift/LOP3 butterfly), parks the
-//     row words in a 32 B-sector buffer and every 256 clocks writes whole
-//     sectors of every instance row (two 16 B stores per row).
+//     one slice word per clock into a ring of NZ z blocks in shared memory;
+//   writer warp c+4 (same SMSP, same TMEM lane quarter): for every 32-clock
+//     block transposes each thread's 32x32 bit tile (PRMT + IMAD-shift/LOP3
+//     butterfly) into tensor memory -- 64 B per row: all 512 columns of the
+//     lane quarter, slot columns permuted by wide_col (keystream.cuh) -- and
+//     every 512 clocks writes 64 B of each of the unit's 1024 rows with
+//     STG.128s of 8 rows x 64 B (tcgen05.ld.16x256b read-back, L2 evict_last).
 //
-// The two are chained by mbarriers (full / empty per z buffer).  The writer's
-// shared-memory and store latencies hide behind the compute warp's LOP3
-// stream instead of stalling it, and the writer's transpose work fills ALU
-// issue slots the compute warp leaves idle.
+// The two are chained by mbarriers (full / empty per z block).  The writer's
+// transposes and its flush bursts run beside the clock loop instead of inside
+// it: the compute warp issues only its cipher logic plus one STS per clock,
+// and the writer's ALU work fills the issue slots a lone clock-loop warp
+// leaves idle.  64 B per row per flush because that is what the DRAM needs
+// (profiles/r2_flush_pattern.log: 32 B per row per flush tops out at 1.4-1.8
+// TB/s for this 1024-rows-per-warp pattern, 64 B reaches 2.9-3.6 TB/s), and
+// one writer per lane quarter is what lets one stream own all 512 columns.
 #pragma once
 #include <cstdint>
 
@@ -27,13 +33,15 @@ namespace ws {
 constexpr int NCOMP = 4;                    // compute warps per CTA (one per SMSP)
 constexpr int BLOCK = 2 * NCOMP * 32;       // + one writer warp each
 constexpr int ZBUF = 32 * 32;               // words in one z block: [t][lane]
-constexpr int PAIR_WORDS = 2 * ZBUF + OS_WORDS;
-constexpr size_t SMEM_BYTES = size_t(NCOMP) * PAIR_WORDS * 4;  // 160 KB
+constexpr int NZ = 4;                       // z blocks in flight per pair (absorb the flush bursts)
+constexpr int PAIR_WORDS = NZ * ZBUF;
+constexpr size_t SMEM_BYTES = size_t(NCOMP) * PAIR_WORDS * 4;  // 64 KB
+constexpr uint32_t NSLOT = 16;              // 32-clock blocks per 64 B row piece
 
 struct Meta {
     uint64_t unit;   // warp-unit of the item (32 groups)
     uint64_t B;      // call-relative index of this 32-clock block
-    uint32_t k_lo;   // first staged sector slot to write on flush
+    uint32_t k_lo;   // first staged slot to write on flush
     uint32_t flags;  // F_FLUSH | F_TERM
 };
 enum : uint32_t { F_FLUSH = 1u, F_TERM = 2u };
@@ -70,25 +78,28 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
     static_assert(32 % U == 0, "U must divide 32");
     constexpr int KB = ks_block<C, U>();
     static_assert(U % KB == 0, "the loop body must hold whole schedule blocks");
-    extern __shared__ uint32_t pair_smem[];  // [NCOMP][2 z blocks + sector buffer]
-    __shared__ uint64_t bar_full[ws::NCOMP][2], bar_empty[ws::NCOMP][2];
-    __shared__ ws::Meta meta[ws::NCOMP][2];
+    extern __shared__ uint32_t pair_smem[];  // [NCOMP][NZ z blocks]
+    __shared__ uint64_t bar_full[ws::NCOMP][ws::NZ], bar_empty[ws::NCOMP][ws::NZ];
+    __shared__ ws::Meta meta[ws::NCOMP][ws::NZ];
     __shared__ uint32_t s_item[ws::NCOMP];
     __shared__ uint64_t s_unit[ws::NCOMP], s_b0[ws::NCOMP];  // per-item context of each compute warp
+    __shared__ uint8_t* s_row0[ws::NCOMP][32];                // writer: row bases of the unit's groups
+    __shared__ uint32_t s_nvalid[ws::NCOMP][32];
+    __shared__ uint32_t s_tmem;
 
     if (threadIdx.x == 0) {
         for (int c = 0; c < ws::NCOMP; ++c)
-            for (int b = 0; b < 2; ++b) {
+            for (int b = 0; b < ws::NZ; ++b) {
                 ws::mbar_init(&bar_full[c][b], 32);
                 ws::mbar_init(&bar_empty[c][b], 32);
             }
     }
-    __syncthreads();
+    // all 512 columns: the writer of lane quarter p owns them for its stream
+    (void)tmem_alloc_cta(&s_tmem, true);  // includes __syncthreads
 
     const uint32_t warp = threadIdx.x >> 5;
     const uint32_t pair = warp % ws::NCOMP;
     uint32_t* zbase = pair_smem + pair * ws::PAIR_WORDS;
-    uint32_t* os = zbase + 2 * ws::ZBUF;
     const uint64_t total = a.units * a.nseg;
 
     if (warp < ws::NCOMP) {
@@ -121,8 +132,8 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
             c.load(a.state, a.Gp, g);
 #pragma unroll 1
             for (uint32_t blk = 0; blk < nblk; ++blk, ++seq) {
-                const uint32_t b = seq & 1u;
-                if (seq >= 2) ws::mbar_wait(&bar_empty[pair][b], ((seq >> 1) - 1) & 1u);
+                const uint32_t b = seq % ws::NZ;
+                if (seq >= ws::NZ) ws::mbar_wait(&bar_empty[pair][b], ((seq / ws::NZ) - 1) & 1u);
                 uint32_t* zb = zbase + b * ws::ZBUF + laneid_volatile();
 #pragma unroll 1
                 for (uint32_t k = 0; k < 32; k += U) {
@@ -134,12 +145,12 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
                 }
                 if (laneid_volatile() == 0) {
                     const uint64_t B = s_b0[pair] + blk;
-                    const uint32_t kk = uint32_t(B & 7);
+                    const uint32_t kk = uint32_t(B % ws::NSLOT);
                     ws::Meta& m = meta[pair][b];
                     m.unit = s_unit[pair];
                     m.B = B;
                     m.k_lo = kk - (blk < kk ? blk : kk);
-                    m.flags = (kk == 7 || blk + 1 == nblk) ? ws::F_FLUSH : 0u;
+                    m.flags = (kk == ws::NSLOT - 1 || blk + 1 == nblk) ? ws::F_FLUSH : 0u;
                 }
                 ws::mbar_arrive(&bar_full[pair][b]);
             }
@@ -157,32 +168,42 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
             }
             next_item(a, slot);
         }
-        const uint32_t b = seq & 1u;
-        if (seq >= 2) ws::mbar_wait(&bar_empty[pair][b], ((seq >> 1) - 1) & 1u);
+        const uint32_t b = seq % ws::NZ;
+        if (seq >= ws::NZ) ws::mbar_wait(&bar_empty[pair][b], ((seq / ws::NZ) - 1) & 1u);
         if (laneid_volatile() == 0) meta[pair][b].flags = ws::F_TERM;
         ws::mbar_arrive(&bar_full[pair][b]);
     } else {
         // ------------------------------------------------------------- writer
         const uint32_t lane = threadIdx.x & 31u;
         for (uint32_t seq = 0;; ++seq) {
-            const uint32_t b = seq & 1u;
-            ws::mbar_wait(&bar_full[pair][b], (seq >> 1) & 1u);
+            const uint32_t b = seq % ws::NZ;
+            ws::mbar_wait(&bar_full[pair][b], (seq / ws::NZ) & 1u);
             const volatile ws::Meta& vm = meta[pair][b];
             const uint32_t flags = vm.flags;
             if (flags & ws::F_TERM) break;
             const uint64_t unit = vm.unit, B = vm.B;
             const uint32_t k_lo = vm.k_lo;
-            const uint32_t k = uint32_t(B & 7);
-            rowmajor_transpose<C::MSB_FIRST>(zbase + b * ws::ZBUF + lane, os + lane, k);
+            const uint32_t k = uint32_t(B % ws::NSLOT);
+            const uint32_t tm = *reinterpret_cast<volatile uint32_t*>(&s_tmem) + (pair << 21);
+            rowmajor_transpose_smem_tmem<C::MSB_FIRST, 16>(zbase + b * ws::ZBUF + lane, tm, wide_col(k));
             ws::mbar_arrive(&bar_empty[pair][b]);
             if (flags & ws::F_FLUSH) {
                 const uint64_t first = (unit * 32u + lane) * 32u;
                 const uint32_t nvalid = first >= a.n ? 0u : uint32_t(a.n - first < 32 ? a.n - first : 32);
                 uint8_t* row0 = static_cast<uint8_t*>(a.out) + (nvalid ? first : 0) * a.row_bytes;
-                rowmajor_store(os + lane, row0, a.row_bytes, nvalid, k_lo, k, (B - (k - k_lo)) * 4);
+                const uint64_t col = (B - (k - k_lo)) * 4;
+                s_row0[pair][lane] = row0;
+                s_nvalid[pair][lane] = nvalid;
+                __syncwarp();
+                if (k_lo == 0 && k == ws::NSLOT - 1 && ((a.row_bytes | col) & 7) == 0 && a.row_bytes < (1ull << 32))
+                    rowmajor_store_tmem_wide(tm, s_row0[pair], s_nvalid[pair], a.row_bytes, col);
+                else
+                    rowmajor_store_tmem_wide_partial(tm, row0, a.row_bytes, nvalid, k_lo, k, col);
+                __syncwarp();
             }
         }
     }
+    tmem_dealloc_cta(*reinterpret_cast<volatile uint32_t*>(&s_tmem), true);
 }
 
 }  // namespace bsk

@@ -145,6 +145,16 @@ def test_mickey_2_40_limit_boundary():
     ("grain", {"rm_tmem": 1, "rm_tma": 0}, 4416 + 256),  # double-buffered staging, progressive flush
     ("mickey2", {"rm_ws": 0, "rm_tmem": 1, "rm_tma": 0}, 2048 + 96),  # ... item ends mid-period
     ("grain", {"rm_tmem": 1, "rm_dbl": 0}, 4416),          # single buffer
+    ("grain", {"rm_wide": 1}, 8192),                      # 64 B staging, whole 512-clock flushes
+    ("grain", {"rm_wide": 1}, 4416),                      # 552 B rows: word-by-word flushes
+    ("grain", {"rm_wide": 1, "seg_clocks": 160}, 2080),   # partial periods at segment ends
+    ("mickey2", {"rm_wide": 1}, 1024 + 512 + 96),
+    ("grain", {"rm_wide": 1, "unroll": 16, "seg_clocks": 1024}, 4096),
+    ("grain", {"rm_l2last": 0}, 8192),                     # evict-first TMA flush
+    ("grain", {"rm_l2last": 0, "rm_tma": 0}, 8192),        # evict-first 8 B sector flush
+    ("grain", {"rm_ws": 1}, 4416),                         # writer warp, 552 B rows (STG.64 pieces)
+    ("grain", {"rm_ws": 1, "seg_clocks": 512}, 4096 + 1024),
+    ("mickey2", {"rm_ws": 1}, 4416),
 ])
 def test_rm_tmem_staging_bit_exact(cipher, opts, bits):
     """ROW_MAJOR with the row segments staged in tensor memory (TMEM) instead

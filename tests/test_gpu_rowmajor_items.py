@@ -30,6 +30,8 @@ RESIDENT_WARPS = 2 * 4 * 148  # whole_units policy: 2 CTAs/SM x 4 clock-loop war
 def _oracle_rows(cipher, keys, ivs, bits):
     if cipher == "mickey2":
         return oracle.mickey2_keystream_batch(keys, ivs, 80, bits)
+    if cipher == "lfsr128":
+        return oracle.lfsr128_keystream_batch(keys, bits)
     return oracle.grain_keystream_batch(keys, ivs, bits)
 
 
@@ -81,6 +83,9 @@ _FORCED = [
     ("grain", {"ctas_per_sm": 1, "seg_clocks": 256, "rm_tmem": 0}, 2048),     # shared-memory staging
     ("mickey2", {"ctas_per_sm": 1, "seg_clocks": 256, "rm_tmem": 0, "rm_ws": 0}, 1024),  # smem staging
     ("mickey2", {"seg_clocks": 256, "rm_ws": 1}, 1024),                        # warp-specialised
+    ("grain", {"rm_wide": 1, "seg_clocks": 1024}, 2048),                      # 64 B staging, lone warps
+    ("lfsr128", {"rm_wide": 1, "seg_clocks": 512}, 2048),                     # 64 B staging
+    ("lfsr128", {"ctas_per_sm": 1, "seg_clocks": 256}, 2048),                 # LFSR default (smem staging)
 ]
 
 
@@ -88,7 +93,8 @@ _FORCED = [
 def test_forced_multi_item_per_warp(cipher, opts, bits):
     n = (1 << 20) + 37  # ragged tail unit
     keys, ivs = inputs.make_inputs(cipher, n, seed=77)
-    kd, vd = torch.from_numpy(keys).cuda(), torch.from_numpy(ivs).cuda()
+    kd = torch.from_numpy(keys).cuda()
+    vd = torch.from_numpy(ivs).cuda() if cipher != "lfsr128" else None
     g = bsrng.Generator(cipher, kd, vd)
     for k, v in opts.items():
         g.set_option(k, v)

@@ -51,11 +51,12 @@ record)
   timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $D/smoke.txt 2>&1
   bench n1_default
   bench n1_reference --impl reference
-  for c in grain aes128ctr lfsr128; do bench c2_$c --cipher $c; done
+  for c in grain aes128ctr; do bench c2_$c --cipher $c --steps 10; done
+  bench c2_lfsr128 --cipher lfsr128 --steps 60
   # paper shape and rekey steps are a few ms: 400+ steps give >= 1 s timed regions
   for c in mickey2 grain aes128ctr; do
-    bench c4_$c --cipher $c --workload c4 --no-cpu-baseline --no-e2e --steps 400 --warmup 20
-    bench rekey_$c --cipher $c --workload rekey --no-cpu-baseline --no-e2e --no-other-mode --steps 400 --warmup 20
+    bench c4_$c --cipher $c --workload c4 --no-cpu-baseline --no-e2e --steps 2000 --warmup 20
+    bench rekey_$c --cipher $c --workload rekey --no-cpu-baseline --no-e2e --no-other-mode --steps 1000 --warmup 20
   done
   bench c3_n1 --workload c3 --steps 3 --warmup 3 --no-other-mode --no-context ;;
 launches)
