@@ -46,10 +46,15 @@ BITS_DEFAULT = 1 << 20
 #  * KERNEL -- what the shipped kernels need: MICKEY 304 with the R reduction
 #    deferred over K = 4-clock blocks (315.5 at K = 2; mickey2.cuh clock_lazy,
 #    DESIGN.md sec. 5 item 10), Grain 37 (+1 to fold into the checksum), AES
-#    17280 (+64 for the checksum XOR tree), LFSR 2 (+0.5 for the checksum).
+#    16848 (MixColumns + AddRoundKey as tools/mc_xor3.py's 84-LOP3 circuit per
+#    column instead of 96; +64 for the checksum XOR tree), LFSR 2 (+0.5 for
+#    the checksum).
 # A kernel whose count is below the algorithmic one can exceed frac = 1.
 MICKEY2_GALOIS_OPS = 327.0
 MICKEY2_OPS_BY_BLOCK = {1: 327.0, 2: 315.5, 4: 304.0}
+# AES kernel count per 32-block encryption: counter + round-0 key 256,
+# SubBytes 10 x 16 x 84, MixColumns + AddRoundKey 9 x 4 x 84, final key 128
+AES_KERNEL_OPS = 256.0 + 10 * 16 * 84 + 9 * 4 * 84 + 128
 ALGORITHMIC_OPS = {"mickey2": 327.0, "grain": 39.0, "aes128ctr": 17280.0 / 128.0, "lfsr128": 2.0}
 
 
@@ -73,7 +78,7 @@ def lop3_per_bit(cipher, mode, unroll=None):
         # feedback XOR4 = 2 LOP3; consume folds the period's output words into
         # the accumulator (0.5 per clock; 128-clock loop body)
         return 2.5 if mode == "consume" else 2.0
-    return (17280.0 + (64.0 if mode == "consume" else 0.0)) / 128.0
+    return (AES_KERNEL_OPS + (64.0 if mode == "consume" else 0.0)) / 128.0
 
 
 CIPHER_NAME = {"mickey2": "MICKEY 2.0", "grain": "Grain v1", "aes128ctr": "AES-128-CTR",

@@ -90,42 +90,27 @@ __device__ __forceinline__ void shift_rows(uint32_t (&s)[128])
     for (int i = 0; i < 128; ++i) s[i] = t[i];
 }
 
-// MixColumns (FIPS-197 5.1.3) + AddRoundKey with round-key row `k` (masks),
-// two LOP3 per output bit.  With u_i = a_i ^ a_{i+1} (indices mod 4):
-//   out_i = 2a_i ^ 3a_{i+1} ^ a_{i+2} ^ a_{i+3} ^ k = a_{i+1} ^ u_{i+2} ^ xtime(u_i) ^ k
-// and xtime(u) = (u << 1) ^ (u_7 ? 0x1b : 0) adds u_7 at significance 0, 1, 3, 4.
-// Byte words are MSB-first: significance s lives at index 7 - s.
+// MixColumns (FIPS-197 5.1.3) + AddRoundKey with round-key row `k` (masks):
+// per column, out_i = 2a_i ^ 3a_{i+1} ^ a_{i+2} ^ a_{i+3} ^ k, a GF(2)-linear
+// map of the column's 32 bit words plus one key word per output.  The
+// program is tools/mc_xor3.py's three-input-XOR circuit (greedy common-
+// subexpression search over 2- and 3-input XOR gates, verified there by
+// simulation and here by the FIPS/SP 800-38A vectors): 84 LOP3 per column,
+// against 96 for the u_i = a_i ^ a_{i+1} form (32 XOR2 for u, then
+// a_{i+1} ^ u_{i+2} ^ xtime(u_i) ^ k as two LOP3 per output bit).
+__device__ __forceinline__ uint32_t x2(uint32_t a, uint32_t b) { return lop3<0x3Cu>(a, b, 0u); }
+__device__ __forceinline__ uint32_t x3(uint32_t a, uint32_t b, uint32_t c) { return lop3<0x96u>(a, b, c); }
 __device__ __forceinline__ void mix_columns_ark(uint32_t (&s)[128], const uint32_t* k)
 {
-    constexpr uint32_t X3 = 0xF0u ^ 0xCCu ^ 0xAAu;  // a ^ b ^ c
-    constexpr uint32_t X2 = 0xF0u ^ 0xCCu;          // a ^ b
 #pragma unroll
     for (int c = 0; c < 4; ++c) {
-        uint32_t u[4][8];
+        uint32_t a[32], o[32];
 #pragma unroll
-        for (int i = 0; i < 4; ++i)
+        for (int j = 0; j < 32; ++j) a[j] = s[32 * c + j];
+        const uint32_t* kk = k + 32 * c;
+#include "aes_mc_lop3.inc"
 #pragma unroll
-            for (int b = 0; b < 8; ++b) u[i][b] = s[8 * (4 * c + i) + b] ^ s[8 * (4 * c + ((i + 1) & 3)) + b];
-        uint32_t o[4][8];
-#pragma unroll
-        for (int i = 0; i < 4; ++i) {
-            const uint32_t* a1 = &s[8 * (4 * c + ((i + 1) & 3))];
-            const uint32_t* kk = &k[8 * (4 * c + i)];
-#pragma unroll
-            for (int sig = 0; sig < 8; ++sig) {
-                const int b = 7 - sig;
-                const uint32_t xt = sig == 0 ? u[i][0] : u[i][b + 1];  // (u << 1) at significance sig
-                const uint32_t t = lop3<X3>(a1[b], u[(i + 2) & 3][b], xt);
-                if (sig == 1 || sig == 3 || sig == 4)
-                    o[i][b] = lop3<X3>(t, u[i][0], kk[b]);  // + u_7 (index 0) from the 0x1b reduction
-                else
-                    o[i][b] = lop3<X2>(t, kk[b], 0u);
-            }
-        }
-#pragma unroll
-        for (int i = 0; i < 4; ++i)
-#pragma unroll
-            for (int b = 0; b < 8; ++b) s[8 * (4 * c + i) + b] = o[i][b];
+        for (int j = 0; j < 32; ++j) s[32 * c + j] = o[j];
     }
 }
 
@@ -137,16 +122,24 @@ __device__ __forceinline__ void add_round_key(uint32_t (&s)[128], const uint32_t
 
 // Counter block for encryption index T (warp-uniform) plus round-0 key:
 // s = (base + T mod 2^128) ^ K0.  base is this thread's sliced initial
-// counter (128 words in shared memory, [b][thread] with stride `st`).
+// counter (128 words in shared memory, [b][thread] with stride `st`, as a
+// shared-window address).  The loads are volatile: hoisted out of the
+// encryption loop, the 128 loop-invariant words spilled 272 B of stack.
 // Bit b has significance 127 - b; the carry ripples from word 127 up.
-__device__ __forceinline__ void counter_block(uint32_t (&s)[128], const uint32_t* base, int st, uint64_t T,
+__device__ __forceinline__ uint32_t lds_volatile(uint32_t saddr)
+{
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(saddr));
+    return v;
+}
+__device__ __forceinline__ void counter_block(uint32_t (&s)[128], uint32_t base, int st, uint64_t T,
                                               const RoundKeys& rk)
 {
     uint32_t c = 0u;
 #pragma unroll
     for (int p = 0; p < 128; ++p) {
         const int b = 127 - p;
-        const uint32_t x = base[b * st];
+        const uint32_t x = lds_volatile(base + 4u * uint32_t(b * st));
         const uint32_t tb = p < 64 ? (uint32_t)0 - (uint32_t)((T >> p) & 1u) : 0u;  // warp-uniform
         s[b] = x ^ c ^ (tb ^ rk.m[0][b]);
         c = (x & c) | ((x | c) & tb);  // majority(x, tb, c)
@@ -167,9 +160,12 @@ __device__ __forceinline__ void counter_block(uint32_t (&s)[128], const uint32_t
 //     carried out of the low five bits.
 // Round key 0 is folded in: the K0 bits >= 5 are XORed into H and H + 1 before
 // the per-bit masks are extracted.
-__device__ __forceinline__ uint32_t bit_mask(uint32_t w, int q)
+template <int Q>
+__device__ __forceinline__ uint32_t bit_mask(uint32_t w)
 {
-    return uint32_t(int32_t(w << (31 - q)) >> 31);  // 0 or ~0
+    // 0 or ~0 = bit Q of w: the shift on the FMA pipe (IMAD.SHL), the sign
+    // broadcast on the ALU pipe
+    return uint32_t(int32_t(shl_fma<31 - Q>(w)) >> 31);
 }
 
 __device__ __forceinline__ void counter_block_lanes(uint32_t (&s)[128], const uint32_t (&V)[4], const RoundKeys& rk,
@@ -182,6 +178,8 @@ __device__ __forceinline__ void counter_block_lanes(uint32_t (&s)[128], const ui
     H[2] = (V[2] >> 5) | (V[1] << 27);
     H[1] = (V[1] >> 5) | (V[0] << 27);
     H[0] = V[0] >> 5;
+    // bits >= 27 of H and H + 1 agree unless bits 0..26 of H are all ones
+    const bool hi_equal = (H[3] & 0x07FFFFFFu) != 0x07FFFFFFu;
     uint32_t cy = 1u;
 #pragma unroll
     for (int w = 3; w >= 0; --w) {
@@ -196,12 +194,21 @@ __device__ __forceinline__ void counter_block_lanes(uint32_t (&s)[128], const ui
     constexpr uint32_t P0[5] = {0xAAAAAAAAu, 0xCCCCCCCCu, 0xF0F0F0F0u, 0xFF00FF00u, 0xFFFF0000u};
 #pragma unroll
     for (int p = 0; p < 5; ++p) s[127 - p] = __funnelshift_r(P0[p], P0[p], c) ^ rk.m[0][127 - p];
-#pragma unroll
-    for (int p = 5; p < 128; ++p) {
-        const int q = p - 5;
-        const uint32_t m0 = bit_mask(H[3 - (q >> 5)], q & 31);
-        const uint32_t m1 = bit_mask(H1[3 - (q >> 5)], q & 31);
-        s[127 - p] = (carry & m1) | (~carry & m0);
+    // lanes j >= 32 - c carried out of the low five bits: they see H + 1
+    static_for<27>([&](auto qq) {
+        constexpr int q = decltype(qq)::value;
+        s[127 - 5 - q] = sel_imm_var(carry, bit_mask<q>(H1[3]), bit_mask<q>(H[3]));
+    });
+    if (hi_equal) {  // the common case: one mask per bit, no select
+        static_for<96>([&](auto qq) {
+            constexpr int q = decltype(qq)::value + 27;
+            s[127 - 5 - q] = bit_mask<q & 31>(H[3 - (q >> 5)]);
+        });
+    } else {
+        static_for<96>([&](auto qq) {
+            constexpr int q = decltype(qq)::value + 27;
+            s[127 - 5 - q] = sel_imm_var(carry, bit_mask<q & 31>(H1[3 - (q >> 5)]), bit_mask<q & 31>(H[3 - (q >> 5)]));
+        });
     }
 }
 
@@ -318,16 +325,23 @@ __global__ void __launch_bounds__(128, 2) aes_ctr_kernel(const __grid_constant__
 #pragma unroll 1
         for (uint32_t e = 0; e < nenc; ++e) {
             uint32_t s[128];
-            aes::counter_block(s, base, 128, T0 + e, rk);
+            aes::counter_block(s, static_cast<uint32_t>(__cvta_generic_to_shared(base)), 128, T0 + e, rk);
             aes::encrypt(s, rk);
             if (LAYOUT == L_CHECKSUM) {
 #pragma unroll
                 for (int b = 0; b < 128; ++b) acc ^= s[b];
             } else if (LAYOUT == L_SLICED) {
                 if (g < a.G) {
-                    uint32_t* o = static_cast<uint32_t*>(a.out) + (bit_begin + uint64_t(e) * 128) * a.G + g;
+                    // one running pointer (IMAD.WIDE on the FMA pipe): 128
+                    // precomputed addresses spilled
+                    uint8_t* o = reinterpret_cast<uint8_t*>(static_cast<uint32_t*>(a.out) +
+                                                            (bit_begin + uint64_t(e) * 128) * a.G + g);
+                    const uint64_t stride = a.G * 4;
 #pragma unroll
-                    for (int b = 0; b < 128; ++b) __stcs(o + uint64_t(b) * a.G, s[b] & m);
+                    for (int b = 0; b < 128; ++b) {
+                        __stcs(reinterpret_cast<uint32_t*>(o), s[b] & m);
+                        o = add_fma(o, stride);
+                    }
                 }
             } else {
                 // four 32-bit tiles: row t of tile k is bit 32k + (t ^ 7) (MSB-first bytes)

@@ -113,6 +113,14 @@ __device__ __forceinline__ uint32_t sel_imm(uint32_t x, uint32_t y)
     return d;
 }
 
+// d = m ? x : y bitwise, m in a register: one LOP3 (0xCA: a ? b : c)
+__device__ __forceinline__ uint32_t sel_imm_var(uint32_t m, uint32_t x, uint32_t y)
+{
+    uint32_t d;
+    asm("lop3.b32 %0, %1, %2, %3, 0xCA;" : "=r"(d) : "r"(m), "r"(x), "r"(y));
+    return d;
+}
+
 template <int S, uint32_t M>
 __device__ __forceinline__ void bt_stage(uint32_t& a, uint32_t& b)
 {
