@@ -73,7 +73,7 @@ captures)
   capture aes_consume aes_ctr --cipher aes128ctr --layout checksum --bits 16384 --reps 2
   capture aes_rowmajor rowmajor_lanes --cipher aes128ctr --layout row_major --bits 16384 --reps 2
   capture lfsr_consume keystream_kernel --cipher lfsr128 --layout checksum --bits 65536 --reps 2
-  capture lfsr_rowmajor keystream_kernel --cipher lfsr128 --layout row_major --bits 32768 --reps 2
+  capture lfsr_rowmajor keystream_rm_ws --cipher lfsr128 --layout row_major --bits 32768 --reps 2
   capture lfsr_sliced keystream_kernel --cipher lfsr128 --layout sliced --bits 65536 --reps 2
   SKIP=0 capture preclock m2_init --layout checksum --bits 32 --reps 1
   SKIP=0 capture grain_init grain_init --cipher grain --layout checksum --bits 32 --reps 1 ;;

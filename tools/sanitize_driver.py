@@ -13,9 +13,14 @@ from paper_conf_icppw_monfaredhkzrg20_b200 import bsrng  # noqa: E402
 
 cases = [
     ("mickey2", 32 * 40 + 9, 1024, {}), ("mickey2", 32 * 32 * 2, 2048, {}),            # TMEM staging, TMA flush
-    ("mickey2", 32 * 40 + 9, 1024, {"rm_tma": 0}), ("mickey2", 32 * 40 + 9, 512, {"rm_ws": 1}),
+    ("mickey2", 32 * 40 + 9, 1024, {"rm_tma": 0}), ("mickey2", 32 * 40 + 9, 1024 + 512, {"rm_ws": 1}),
+    ("mickey2", 32 * 40 + 9, 1024, {"rm_wide": 1}), ("mickey2", 32 * 40 + 9, 1024, {"rm_l2last": 0}),
     ("grain", 32 * 40 + 9, 1024, {}), ("grain", 32 * 32 * 2, 2048, {}), ("grain", 32 * 40, 552 * 8, {}),
-    ("aes128ctr", 32 * 9 + 5, 4480, {}), ("lfsr128", 32 * 37 + 13, 1024, {}),
+    ("grain", 32 * 40 + 9, 2048, {"rm_ws": 1}), ("grain", 32 * 40, 552 * 8, {"rm_ws": 1}),
+    ("grain", 32 * 40 + 9, 1024 + 512, {"rm_wide": 1}), ("grain", 32 * 40 + 9, 1024, {"rm_tma": 0}),
+    ("aes128ctr", 32 * 9 + 5, 4480, {}), ("aes128ctr", 32 * 9 + 5, 4480, {"rm_ws": 0}),
+    ("lfsr128", 32 * 37 + 13, 1024, {}), ("lfsr128", 32 * 37 + 13, 2048 + 96, {}),
+    ("lfsr128", 32 * 37 + 13, 1024, {"rm_ws": 0}),
 ]
 # SANITIZE_NO_TMEM=1: shared-memory staging instead of tensor memory (synccheck
 # reports tcgen05.alloc's shared-memory result slot as an uninitialised barrier)
