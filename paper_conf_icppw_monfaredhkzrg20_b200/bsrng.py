@@ -14,7 +14,8 @@ import numpy as np
 from . import inputs as _inputs
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libbsrng.so")
+# BSRNG_LIB: an alternative build of the same library (A/B runs of kernel variants)
+LIB_PATH = os.environ.get("BSRNG_LIB") or os.path.join(_PKG, "libbsrng.so")
 
 MICKEY2, GRAIN_V1, AES128_CTR, LFSR128 = 1, 2, 3, 4
 ROW_MAJOR, SLICED, CHECKSUM = 0, 1, 2

@@ -31,7 +31,7 @@ def _sources():
 
 def _compile(unit: str, objdir: str, verbose: bool) -> str:
     obj = os.path.join(objdir, unit.replace(".cu", ".o"))
-    cmd = [NVCC, *FLAGS, "-Xptxas", "-v", "-c", "-o", obj, os.path.join(CSRC, unit)]
+    cmd = [NVCC, *FLAGS, *_DEFINES, "-Xptxas", "-v", "-c", "-o", obj, os.path.join(CSRC, unit)]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         sys.stderr.write(r.stdout + r.stderr)
@@ -41,11 +41,14 @@ def _compile(unit: str, objdir: str, verbose: bool) -> str:
     return obj
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
+def build(force: bool = False, verbose: bool = False, out: str = LIB, defines=()) -> str:
+    """Compile libbsrng.so (or `out`, with extra -D `defines`, for A/B builds)."""
     srcs = _sources()
-    if (not force and os.path.exists(LIB)
+    if (not force and not defines and out == LIB and os.path.exists(LIB)
             and all(os.path.getmtime(LIB) >= os.path.getmtime(s) for s in srcs)):
         return LIB
+    global _DEFINES
+    _DEFINES = [f"-D{d}" for d in defines]
     objdir = os.path.join(CSRC, f".obj{os.getpid()}")
     os.makedirs(objdir, exist_ok=True)
     try:
@@ -53,18 +56,22 @@ def build(force: bool = False, verbose: bool = False) -> str:
         # submitting it first keeps the wall time at its compile time
         with ThreadPoolExecutor(max_workers=len(UNITS)) as ex:
             objs = list(ex.map(lambda u: _compile(u, objdir, verbose), UNITS))
-        tmp = LIB + f".tmp{os.getpid()}"
+        tmp = out + f".tmp{os.getpid()}"
         r = subprocess.run([NVCC, *ARCH, "-shared", "-o", tmp, *objs], capture_output=True, text=True)
         if r.returncode != 0:
             sys.stderr.write(r.stdout + r.stderr)
             raise RuntimeError("nvcc failed linking libbsrng.so")
-        os.replace(tmp, LIB)
+        os.replace(tmp, out)
     finally:
         for f in os.listdir(objdir):
             os.remove(os.path.join(objdir, f))
         os.rmdir(objdir)
-    return LIB
+    return out
 
+
+_DEFINES: list = []
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))
+    defs = [a[2:] for a in sys.argv[1:] if a.startswith("-D")]
+    outs = [a[6:] for a in sys.argv[1:] if a.startswith("--out=")]
+    print(build(force="--force" in sys.argv, verbose="-v" in sys.argv, out=outs[0] if outs else LIB, defines=defs))

@@ -37,6 +37,9 @@ constexpr int NZ = 4;                       // z blocks in flight per pair (abso
 constexpr int PAIR_WORDS = NZ * ZBUF;
 constexpr size_t SMEM_BYTES = size_t(NCOMP) * PAIR_WORDS * 4;  // 64 KB
 constexpr uint32_t NSLOT = 16;              // 32-clock blocks per 64 B row piece
+#ifndef WRITER_SLEEP_NS
+#define WRITER_SLEEP_NS 200
+#endif
 
 struct Meta {
     uint64_t unit;   // warp-unit of the item (32 groups)
@@ -68,6 +71,26 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity)
         "@!p bra WAIT_%=;\n\t}" ::"r"(smem_u32(bar)),
         "r"(parity)
         : "memory");
+}
+
+// The writer's wait for a full z block: it is the faster side and usually
+// finds the block not yet full; a tight try_wait loop keeps it eligible every
+// cycle and takes issue slots from the clock-loop warp on the same SMSP (ncu:
+// the writer's spin branch was executed ~75x per block), so it backs off.
+__device__ __forceinline__ void mbar_wait_sleepy(uint64_t* bar, uint32_t parity)
+{
+    uint32_t ok;
+    for (;;) {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\t"
+            "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}"
+            : "=r"(ok)
+            : "r"(smem_u32(bar)), "r"(parity)
+            : "memory");
+        if (ok) break;
+        __nanosleep(WRITER_SLEEP_NS);
+    }
 }
 
 }  // namespace ws
@@ -177,7 +200,7 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
         const uint32_t lane = threadIdx.x & 31u;
         for (uint32_t seq = 0;; ++seq) {
             const uint32_t b = seq % ws::NZ;
-            ws::mbar_wait(&bar_full[pair][b], (seq / ws::NZ) & 1u);
+            ws::mbar_wait_sleepy(&bar_full[pair][b], (seq / ws::NZ) & 1u);
             const volatile ws::Meta& vm = meta[pair][b];
             const uint32_t flags = vm.flags;
             if (flags & ws::F_TERM) break;

@@ -110,3 +110,55 @@ def test_forced_multi_item_per_warp(cipher, opts, bits):
     want = _oracle_rows(cipher, keys[idx], ivs[idx], 2 * bits)
     assert np.array_equal(got[0], want[:, : bits // 8])
     assert np.array_equal(got[1], want[:, bits // 8:])
+
+
+@pytest.mark.parametrize("cipher", ["lfsr128", "aes128ctr"])
+def test_bench_materialise_shape_other_ciphers(cipher):
+    """The LFSR (writer-warp kernel, 64 B TMEM staging) and AES-128-CTR
+    (block-lane kernel) at the bench's materialise shape: n = 2^22, two
+    consecutive 2^15-bit ROW_MAJOR calls, sampled rows vs the oracle."""
+    n, chunk = 1 << 22, 1 << 15
+    keys, ivs = inputs.make_inputs(cipher, n)
+    if cipher == "aes128ctr":
+        key = inputs.aes_key()
+        g = bsrng.Generator(cipher, torch.from_numpy(key).cuda(), torch.from_numpy(ivs).cuda())
+    else:
+        g = bsrng.Generator(cipher, torch.from_numpy(keys).cuda(), None)
+    buf = torch.empty(g.out_bytes(chunk, "row_major"), dtype=torch.uint8, device="cuda")
+    units = n // 1024
+    rng = np.random.default_rng(22)
+    idx = _sample_rows(n, [0, 1, 591, 592, 1183, 1184, 2368, units - 1], rng)
+    got = []
+    for _ in range(2):
+        g.generate(buf, chunk, "row_major")
+        torch.cuda.synchronize()
+        got.append(_gather_rows(buf, idx, chunk // 8))
+    if cipher == "aes128ctr":
+        want = oracle.aes128_ctr_keystream_batch(bytes(inputs.aes_key()), ivs[idx], 2 * chunk)
+    else:
+        want = oracle.lfsr128_keystream_batch(keys[idx], 2 * chunk)
+    assert np.array_equal(got[0], want[:, : chunk // 8])
+    assert np.array_equal(got[1], want[:, chunk // 8:])
+
+
+@pytest.mark.parametrize("cipher", ["grain", "mickey2", "lfsr128"])
+def test_paper_shape_rowmajor_sampled(cipher):
+    """configs[3]: 2^19 instances x 4416 clocks (552 B rows, 8 B aligned) in
+    the launch configuration bench.py times (Grain and the LFSR: writer-warp
+    kernel with two STG.64 per 16 B piece; MICKEY: double-buffered TMEM), two
+    calls, sampled rows vs the oracle."""
+    n, bits = 1 << 19, 4416
+    keys, ivs = inputs.make_inputs(cipher, n, seed=3)
+    g = bsrng.Generator(cipher, torch.from_numpy(keys).cuda(),
+                        None if cipher == "lfsr128" else torch.from_numpy(ivs).cuda())
+    buf = torch.empty(g.out_bytes(bits, "row_major"), dtype=torch.uint8, device="cuda")
+    rng = np.random.default_rng(4)
+    idx = _sample_rows(n, [0, 1, 255, 256, 511], rng, extra=160)
+    got = []
+    for _ in range(2):
+        g.generate(buf, bits, "row_major")
+        torch.cuda.synchronize()
+        got.append(_gather_rows(buf, idx, bits // 8))
+    want = _oracle_rows(cipher, keys[idx], ivs[idx], 2 * bits)
+    assert np.array_equal(got[0], want[:, : bits // 8])
+    assert np.array_equal(got[1], want[:, bits // 8:])
