@@ -85,7 +85,8 @@ sanitize)
 micro)
   (cd tools/microbench && ./alu_peak 200000 && ./curand_bench 4294967296 && ./write_peak) > $D/micro.log 2>&1 ;;
 sweep)
-  timeout 2400 python tools/sweep_c5.py > $D/sweep.jsonl 2> $D/sweep.err ;;
+  timeout 2400 python tools/sweep_c5.py > $D/sweep.jsonl 2> $D/sweep.err
+  (cd tools/microbench && timeout 300 ./curand_bench 2147483648 && timeout 300 ./curand_bench 17179869184) > $D/curand.log 2>&1 ;;
 *)
   echo "unknown command $cmd"; exit 2 ;;
 esac

@@ -8,8 +8,11 @@ Sweeps, for bitsliced MICKEY 2.0 (and a slice for Grain v1 / AES-128-CTR):
     SMSP (`ctas_per_sm` 1/2) vs the auto policy;
   * instances n in {2^19 (the paper's 64x256x32), 2^22, 2^25};
   * clocks per launch in {4416, 12992 (PAPER.md:751-755), 2^16, 2^20};
-  * clocks unrolled per loop iteration U (register renaming vs I-cache);
-  * output layout (consume / SLICED / ROW_MAJOR, plain vs warp-specialised).
+  * output layout (consume / SLICED / ROW_MAJOR) and the ROW_MAJOR staging
+    variants (TMEM + TMA flush, TMEM + 8 B stores, shared memory, writer warps
+    with 64 B TMEM staging, a lone warp with 64 B staging) for MICKEY, Grain
+    and the LFSR.  (Round 1 also swept MICKEY's unroll U in {2, 4, 8}; only
+    U = 4 is built since round 2: profiles/r1_sweep_c5.md.)
 Every point is CUDA-event timed on a warmed stream (best of `--reps`), with the
 algorithmic LOP3 rate against the ALU roofline at the SM clock sampled by
 nvidia-smi during the run.  cuRAND on the same byte count is timed by
@@ -32,8 +35,9 @@ import torch  # noqa: E402
 
 from paper_conf_icppw_monfaredhkzrg20_b200 import bsrng  # noqa: E402
 
-OPS = {"mickey2": 304.0,  # deferred R reduction (327 in Galois form)
-       "grain": 37.0, "aes128ctr": 17280.0 / 128.0}
+OPS = {"mickey2": 304.0,  # kernel count: deferred R reduction (327 in Galois form)
+       "grain": 37.0, "aes128ctr": 16848.0 / 128.0, "lfsr128": 2.0}
+ALG = {"mickey2": 327.0, "grain": 39.0, "aes128ctr": 17280.0 / 128.0, "lfsr128": 2.0}
 PAPER_CLOCKS = (4416, 12992)  # multiples of 32 nearest the paper's 4,400 / 13,000
 
 
@@ -97,7 +101,9 @@ def point(cipher, n, bits, layout, opts, reps, chunk=None, nsm=148):
     ops = per_clock * (n / 32) * bits / (best * 1e-3)
     peak = nsm * 64 * mhz * 1e6
     return {"cipher": cipher, "n": n, "clocks_per_call": chunk, "clocks": bits, "layout": layout, "opts": opts,
-            "ms": round(best, 3), "tbps": round(tbps, 4), "sm_mhz": mhz, "alu_frac": round(ops / peak, 4)}
+            "ms": round(best, 3), "tbps": round(tbps, 4), "sm_mhz": mhz, "alu_frac": round(ops / peak, 4),
+            "alu_frac_alg": round(ALG[cipher] * (n / 32) * bits / (best * 1e-3) / peak, 4),
+            "hbm_write_gbs": round(n * bits / 8 / (best * 1e-3) / 1e9, 1) if layout == "row_major" else None}
 
 
 def main():
@@ -123,18 +129,21 @@ def main():
                 emit(d)
     if a.quick:
         return
-    # 2. clocks unrolled per loop iteration (C2 shape, 2^16 clocks)
-    for u in (2, 4, 8):
-        for lay in ("checksum", "row_major"):
-            d = point("mickey2", 1 << 22, 1 << 16, lay, {"unroll": u}, a.reps,
-                      chunk=(1 << 15) if lay == "row_major" else None, nsm=nsm)
-            d["sweep"] = "unroll"
-            emit(d)
-    # 3. output layouts, ROW_MAJOR plain vs warp-specialised, staging chunk
-    for lay, o in [("checksum", {}), ("sliced", {}), ("row_major", {"rm_ws": 0}), ("row_major", {"rm_ws": 1})]:
-        for chunk in ((1 << 12, 1 << 15) if lay != "checksum" else (1 << 16,)):
-            d = point("mickey2", 1 << 22, 1 << 16, lay, o, a.reps, chunk=chunk, nsm=nsm)
+    # 2. output layouts (MICKEY, C2 shape, 2^16 clocks per instance)
+    for lay, chunks in [("checksum", (1 << 16,)), ("sliced", (1 << 12, 1 << 15)), ("row_major", (1 << 12, 1 << 15))]:
+        for chunk in chunks:
+            d = point("mickey2", 1 << 22, 1 << 16, lay, {}, a.reps, chunk=chunk, nsm=nsm)
             d["sweep"] = "layout"
+            emit(d)
+    # 3. ROW_MAJOR staging variants (2^15-bit calls, 4 KB rows)
+    variants = [("tmem_tma", {"rm_ws": 0, "rm_tmem": 1}), ("tmem_8B", {"rm_ws": 0, "rm_tmem": 1, "rm_tma": 0}),
+                ("tmem_evict_first", {"rm_ws": 0, "rm_tmem": 1, "rm_l2last": 0}),
+                ("smem", {"rm_ws": 0, "rm_tmem": 0}), ("writer_warps_64B", {"rm_ws": 1}),
+                ("lone_warp_64B", {"rm_ws": 0, "rm_wide": 1})]
+    for cipher, bits in (("mickey2", 1 << 16), ("grain", 1 << 17), ("lfsr128", 1 << 18)):
+        for name, o in variants:
+            d = point(cipher, 1 << 22, bits, "row_major", o, a.reps, chunk=1 << 15, nsm=nsm)
+            d["sweep"], d["staging"] = "rm_staging", name
             emit(d)
     # 4. Grain v1 and AES-128-CTR: occupancy and unroll at the C2 shape
     for cipher, opts in [("grain", [{"ctas_per_sm": 1}, {"ctas_per_sm": 2}, {"unroll": 16}, {}]),

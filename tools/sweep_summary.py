@@ -32,17 +32,22 @@ def main():
         out.append("")
     for sw, title in (("unroll", "Clocks unrolled per loop iteration U (MICKEY 2.0, n = 2^22, 2^16 clocks)"),
                       ("layout", "Output layouts (MICKEY 2.0, n = 2^22, 2^16 clocks)"),
+                      ("rm_staging", "ROW_MAJOR staging variants (n = 2^22, 2^15-bit calls = 4 KB rows)"),
                       ("cipher", "Grain v1 / AES-128-CTR occupancy and unroll (n = 2^22, 2^16 clocks)")):
         sel = [r for r in rows if r.get("sweep") == sw]
         if not sel:
             continue
         out.append(f"### {title}\n")
-        out.append("| cipher | layout | clocks/call | options | ms | Tb/s | ALU frac | SM MHz |")
-        out.append("|---|---|---|---|---|---|---|---|")
+        out.append("| cipher | layout | clocks/call | options | ms | Tb/s | ALU frac (kernel ops) | ALU frac (sec. 8(d) ops) | HBM writes GB/s | SM MHz |")
+        out.append("|---|---|---|---|---|---|---|---|---|---|")
         for r in sel:
-            opts = ", ".join(f"{k}={v}" for k, v in r["opts"].items()) or "default"
+            opts = (r.get("staging", "") + ": " if r.get("staging") else "") + \
+                (", ".join(f"{k}={v}" for k, v in r["opts"].items()) or "default")
+            alg = r.get("alu_frac_alg")
+            hbm = r.get("hbm_write_gbs")
             out.append(f"| {r['cipher']} | {r['layout']} | {r['clocks_per_call']} | {opts} | {r['ms']} | "
-                       f"{r['tbps']:.3f} | {r['alu_frac']:.3f} | {r['sm_mhz']} |")
+                       f"{r['tbps']:.3f} | {r['alu_frac']:.3f} | {alg if alg is not None else '-'} | "
+                       f"{hbm if hbm is not None else '-'} | {r['sm_mhz']} |")
         out.append("")
     if len(sys.argv) > 2:
         out.append("### cuRAND on the same B200 (context)\n")
