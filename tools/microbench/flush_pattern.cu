@@ -16,7 +16,7 @@
 #include <cstdint>
 #include <cstdio>
 
-enum { QUAD_G, QUAD_Q, PAIR_G, PAIR_Q, ONE, SEG64, SEG128, SEG256 };
+enum { QUAD_G, QUAD_Q, PAIR_G, PAIR_Q, ONE, SEG64, SEG128, SEG256, MIX };
 // store cache policy: 0 = evict-first (st.global.cs), 1 = default (write-back,
 // L2 evict_normal), 2 = L2 evict_last (createpolicy)
 template <int POL>
@@ -87,6 +87,24 @@ __global__ void __launch_bounds__(128) flush_kernel(uint8_t* out, uint64_t pitch
                     uint8_t* p = base + uint64_t(row) * pitch + c + 16 * (lane & 1);
                     st128<POL>(p, make_uint4(v, it, lane, 1));
                 }
+            } else if (V == MIX) {
+                // warps 0-3 of each 8-warp SM: 64 B per row per flush (4 lanes x
+                // 16 B, 8 rows per STG.128); warps 4-7: 32 B (4 lanes x 8 B)
+                const bool wide = (blockIdx.x & 1) == 0;  // 2 CTAs per SM: one wide, one narrow
+                if (wide) {
+                    if (c % 64) continue;
+#pragma unroll 4
+                    for (uint32_t it = 0; it < 128; ++it) {
+                        const uint32_t row = it * 8 + (lane >> 2);
+                        st128<POL>(base + uint64_t(row) * pitch + c + 16 * (lane & 3), make_uint4(v, it, lane, 3));
+                    }
+                } else {
+#pragma unroll 4
+                    for (uint32_t it = 0; it < 128; ++it) {
+                        const uint32_t row = it * 8 + (lane >> 2);
+                        st64<POL>(base + uint64_t(row) * pitch + c + 8 * (lane & 3), make_uint2(v, it));
+                    }
+                }
             } else if (V >= SEG64) {
                 // BPR bytes per row per flush (c advances by BPR), 16 B per lane:
                 // one instruction = 512 / BPR consecutive rows x BPR contiguous bytes
@@ -156,6 +174,10 @@ int main()
             run<SEG128, 0>("seg128", buf, pitch, units, sms, ctas);
             run<SEG128, 2>("seg128", buf, pitch, units, sms, ctas);
             run<SEG256, 0>("seg256", buf, pitch, units, sms, ctas);
+            if (ctas == 2) {
+                run<MIX, 0>("mix_64_32", buf, pitch, units, sms, ctas);
+                run<MIX, 2>("mix_64_32", buf, pitch, units, sms, ctas);
+            }
         }
     }
     cudaFree(buf);
