@@ -108,7 +108,9 @@ uint64_t max_bits(bsrng_cipher c) { return c == BSRNG_MICKEY2 ? (1ull << 40) : (
 // the NULL / legacy / per-thread streams then resolve to that device).
 int check_stream(const bsrng_t* h, cudaStream_t st)
 {
-    if (!st) return BSRNG_OK;
+    // NULL and the special legacy / per-thread handles name the current
+    // device's stream, which the caller's DeviceGuard made the handle's
+    if (!st || st == cudaStreamLegacy || st == cudaStreamPerThread) return BSRNG_OK;
     int sdev = -1;
     cudaError_t e = cudaStreamGetDevice(st, &sdev);
     if (e != cudaSuccess) {

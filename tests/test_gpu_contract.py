@@ -130,6 +130,11 @@ def test_stream_of_the_handles_device_is_accepted():
     buf = torch.zeros(1, dtype=torch.int64, device="cuda:0")
     g.generate(buf, 256, "checksum", stream=st)
     st.synchronize()
+    # the special handles cudaStreamLegacy (1) and cudaStreamPerThread (2)
+    L = bsrng.lib()
+    for special in (1, 2):
+        assert L.bsrng_generate(g.handle, buf.data_ptr(), 256, bsrng.CHECKSUM, special) == bsrng.OK, bsrng.last_error()
+    torch.cuda.synchronize()
 
 
 @pytest.mark.skipif(not torch.cuda.is_available() or torch.cuda.device_count() < 2,
