@@ -540,6 +540,24 @@ def run_ours(args, rank, world, local_rank):
                "traffic": None}
         if clocks and clocks.get("sm_mhz"):
             out["frac_at_sampled_clock"] = alg * units / (nsm * ALU_LANES_PER_SM_CLK * clocks["sm_mhz"] * 1e6 / 1e12)
+        if mode == "materialise":
+            # roofline choice by arithmetic intensity: LOP3 per byte written
+            # (4 B per group-clock) against the ridge = LOP3 peak / HBM peak.
+            # The LFSR's 2 LOP3 per 4 B sit far left of the ridge: its ROW_MAJOR
+            # line is bound by HBM writes, the other ciphers' by the ALU.
+            hbm = float(peaks.get("hbm_gbs", 6467.7))
+            intensity = alg / 4.0
+            ridge = peak * 1e12 / (hbm * 1e9)
+            wr_gbs = units * 1e12 * 4 / 1e9  # bytes written per s
+            out["lop3_per_byte"] = intensity
+            out["ridge_lop3_per_byte"] = ridge
+            out["hbm_write_gbs"] = wr_gbs
+            out["hbm_frac"] = wr_gbs / hbm
+            if intensity < ridge:
+                out.update({"bound": "hbm", "achieved": wr_gbs, "peak": hbm, "unit": "GB/s",
+                            "frac": wr_gbs / hbm,
+                            "alu_frac": alg * units / peak,
+                            "peak_basis": "MEASURED_PEAKS.json hbm_gbs (copy bandwidth, read + write)"})
         return out
 
     results = {}
