@@ -675,24 +675,43 @@ __device__ __forceinline__ void rowmajor_store_tmem_wide(uint32_t tm, uint8_t* c
     }
 }
 
-// Partial 64 B flush: slots [k_lo, k_hi] of this thread's own rows, word by
-// word (item boundaries that are not whole 512-clock periods, rows that are
-// not 16 B aligned).  The 32x32b loads are warp-collective: every lane runs them.
-__device__ __forceinline__ void rowmajor_store_tmem_wide_partial(uint32_t tm, uint8_t* row0, uint64_t row_bytes,
-                                                                 uint32_t nvalid, uint32_t k_lo, uint32_t k_hi,
-                                                                 uint64_t col)
+// Partial 64 B flush: slots [k_lo, k_hi] only (item boundaries that are not
+// whole 512-clock periods, e.g. the paper shape's 4416 clocks = 8 periods + 10
+// slots; rows that are only 4 B aligned).  Same 16x256b read-back as the
+// whole flush, one predicated 4 B store per slot: each store instruction
+// covers 8 rows x 4 slots, instead of 32 rows x 1 slot from each thread's own
+// rows (the first version wrote the paper shape's last 10 slots that way).
+__device__ __forceinline__ void rowmajor_store_tmem_wide_partial(uint32_t tm, uint8_t* const* row0s,
+                                                                 const uint32_t* nvalids, uint64_t row_bytes,
+                                                                 uint32_t k_lo, uint32_t k_hi, uint64_t col)
 {
     tmem_wait_st();
-    uint8_t* p = row0 + col;
+    const uint32_t t = laneid_volatile();
+    const uint32_t j = t & 3u;
 #pragma unroll 1
-    for (uint32_t q = 0; q < 32; ++q) {
-        uint32_t v[16];  // v[wide_col(k)] = slot k of row q
-        tmem_ld16(tm + q * 16, v);
-        if (q < nvalid) {
+    for (uint32_t h = 0; h < 2; ++h) {
+        const uint32_t la = 16 * h + (t >> 2), lb = la + 8;
+        uint8_t* pa = row0s[la] + col;
+        uint8_t* pb = row0s[lb] + col;
+        const uint32_t na = nvalids[la], nb = nvalids[lb];
+#pragma unroll 1
+        for (uint32_t q = 0; q < 32; q += 2) {
+            uint32_t v[16];
+            tmem_ld16x256b_x4(tm + ((16 * h) << 16) + q * 16, v);
 #pragma unroll
-            for (int k = 0; k < 16; ++k)
-                if (uint32_t(k) >= k_lo && uint32_t(k) <= k_hi)
-                    __stcs(reinterpret_cast<uint32_t*>(p + q * row_bytes) + (k - k_lo), v[wide_col(k)]);
+            for (int r = 0; r < 2; ++r) {
+#pragma unroll
+                for (int m = 0; m < 4; ++m) {
+                    // slot 4j + m sits in v[8r + (m & 1) + (m & 2 ? 4 : 0)] (lane la), +2 (lane lb)
+                    const int iv = 8 * r + (m & 1) + ((m & 2) ? 4 : 0);
+                    const uint32_t sl = 4 * j + m;
+                    if (sl >= k_lo && sl <= k_hi) {
+                        if (q + r < na) __stcs(reinterpret_cast<uint32_t*>(pa + (q + r) * row_bytes) + (sl - k_lo), v[iv]);
+                        if (q + r < nb)
+                            __stcs(reinterpret_cast<uint32_t*>(pb + (q + r) * row_bytes) + (sl - k_lo), v[iv + 2]);
+                    }
+                }
+            }
         }
     }
 }
@@ -1011,8 +1030,8 @@ __global__ void __launch_bounds__(BLOCK) keystream_kernel(const __grid_constant_
                                 rowmajor_store_tmem_wide(tm_addr(), s_row0 + (t & ~31u), s_nvalid + (t & ~31u),
                                                          a.row_bytes, col);
                             else
-                                rowmajor_store_tmem_wide_partial(tm_addr(), s_row0[t], a.row_bytes, s_nvalid[t],
-                                                                 k_lo, k, col);
+                                rowmajor_store_tmem_wide_partial(tm_addr(), s_row0 + (t & ~31u),
+                                                                 s_nvalid + (t & ~31u), a.row_bytes, k_lo, k, col);
                         } else if (DBL && k_lo == 0 && k == 7 && blk + 1 < nblk && full_real &&
                             ((a.row_bytes | col) & 7) == 0) {
                             // flushed during the next period (other buffer)

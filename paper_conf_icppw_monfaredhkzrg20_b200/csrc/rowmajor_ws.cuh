@@ -221,7 +221,7 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
                 if (k_lo == 0 && k == ws::NSLOT - 1 && ((a.row_bytes | col) & 7) == 0 && a.row_bytes < (1ull << 32))
                     rowmajor_store_tmem_wide(tm, s_row0[pair], s_nvalid[pair], a.row_bytes, col);
                 else
-                    rowmajor_store_tmem_wide_partial(tm, row0, a.row_bytes, nvalid, k_lo, k, col);
+                    rowmajor_store_tmem_wide_partial(tm, s_row0[pair], s_nvalid[pair], a.row_bytes, k_lo, k, col);
                 __syncwarp();
             }
         }
