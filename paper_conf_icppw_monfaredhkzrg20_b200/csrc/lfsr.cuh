@@ -24,7 +24,7 @@ struct Lfsr128 {
     static constexpr bool RM_TMEM = false, RM_SEGMENTED = true;
     // ROW_MAJOR: always the warp-specialised kernel with 64 B TMEM staging per
     // row (rowmajor_ws.cuh): 2 LOP3 per clock leave the output path as the
-    // whole cost, and 64 B per row per flush is what the DRAM needs (C2 25.4
+    // whole cost, and 64 B per row per flush is what the DRAM needs (C2 26.4
     // vs 11.9 Tb/s with 32 B smem staging)
     static constexpr int RM_WS = 2;
     // consume: one 128-clock body (the rotation period), no moves (keystream.cuh)
@@ -70,6 +70,21 @@ struct Lfsr128 {
         acc = lop3<0x96u>(lop3<0x96u>(p[0], p[1], p[2]), p[3], p[4]);
 #pragma unroll
         for (int t = 0; t < 128; ++t)
+            s[t] = lop3<0x96u>(lop3<0x96u>(s[(t + 29) & 127], s[(t + 27) & 127], s[(t + 2) & 127]), s[t], 0u);
+    }
+    // ROW_MAJOR period body (rowmajor_ws.cuh), block J = clocks 32J..32J+31
+    // of a 128-clock period: their outputs are the entry state words
+    // s[32J..32J+31] (handed to put(u, word)), after which those registers are
+    // clocked in place as in consume_period (registers of later blocks still
+    // hold their entry words when their block comes).  No moves.
+    static constexpr int PERIOD_BLOCKS = 4;
+    template <int J, class F>
+    __device__ __forceinline__ void period_block(F&& put)
+    {
+#pragma unroll
+        for (int u = 0; u < 32; ++u) put(u, s[32 * J + u]);
+#pragma unroll
+        for (int t = 32 * J; t < 32 * J + 32; ++t)
             s[t] = lop3<0x96u>(lop3<0x96u>(s[(t + 29) & 127], s[(t + 27) & 127], s[(t + 2) & 127]), s[t], 0u);
     }
     __device__ __forceinline__ void clock()

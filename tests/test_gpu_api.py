@@ -18,13 +18,15 @@ def _want(cipher, keys, ivs, bits, first_block=0):
         return oracle.mickey2_keystream_batch(keys, ivs, 80, bits)
     if cipher == "grain":
         return oracle.grain_keystream_batch(keys, ivs, bits)
+    if cipher == "lfsr128":
+        return oracle.lfsr128_keystream_batch(keys, bits)
     return oracle.aes128_ctr_keystream_batch(bytes(inputs.aes_key()), ivs, bits, first_block=first_block)
 
 
 def _gen(cipher, keys, ivs, **kw):
     if cipher == "aes128ctr":
         return bsrng.Generator(cipher, inputs.aes_key(), ivs, **kw)
-    return bsrng.Generator(cipher, keys, ivs, **kw)
+    return bsrng.Generator(cipher, keys, None if cipher == "lfsr128" else ivs, **kw)
 
 
 @pytest.mark.parametrize("cipher", ["mickey2", "grain", "aes128ctr"])
@@ -58,6 +60,7 @@ def test_zero_bits_is_noop(cipher):
     ("grain", {"rm_tmem": 0, "ctas_per_sm": 2, "seg_clocks": 384}),
     ("mickey2", {"rm_ws": 0, "rm_tmem": 0}), ("mickey2", {"rm_ws": 0, "rm_tmem": 0, "seg_clocks": 160}),
     ("aes128ctr", {"ctas_per_sm": 1}), ("aes128ctr", {"rm_ws": 0}), ("aes128ctr", {"seg_clocks": 4096}),
+    ("lfsr128", {}), ("lfsr128", {"rm_ws": 1, "seg_clocks": 512}), ("lfsr128", {"seg_clocks": 1536}),
 ])
 def test_options_stay_bit_exact(cipher, opts):
     n, bits = 32 * 40 + 9, 8192
@@ -155,6 +158,11 @@ def test_mickey_2_40_limit_boundary():
     ("grain", {"rm_ws": 1}, 4416),                         # writer warp, 552 B rows (STG.64 pieces)
     ("grain", {"rm_ws": 1, "seg_clocks": 512}, 4096 + 1024),
     ("mickey2", {"rm_ws": 1}, 4416),
+    # LFSR writer-warp kernel: 128-clock period bodies plus per-clock remainders
+    ("lfsr128", {}, 8192),
+    ("lfsr128", {}, 4416),                                # 34.5 periods; 552 B rows
+    ("lfsr128", {"seg_clocks": 512}, 4096 + 1024 + 96),   # items of 4 periods, remainder block
+    ("lfsr128", {"seg_clocks": 1056}, 3168 + 32),         # items of 33 blocks: mid-flush-period starts
 ])
 def test_rm_tmem_staging_bit_exact(cipher, opts, bits):
     """ROW_MAJOR with the row segments staged in tensor memory (TMEM) instead

@@ -1,9 +1,8 @@
-D=gpurun_out/ab5; mkdir -p $D
-for v in base fma16; do
-  if [ $v = fma16 ]; then export BSRNG_LIB=$PWD/build/libbsrng_fma16.so; else unset BSRNG_LIB; fi
-  run() { name=$1; shift; timeout 300 python bench.py --no-context --no-cpu-baseline --no-e2e --warmup 3 --mode materialise --no-other-mode "$@" > $D/${v}_$name.json 2>$D/${v}_$name.err; }
-  run grain_c2 --cipher grain --steps 8
-  run mickey_c2 --cipher mickey2 --steps 3 --bits 131072
-  run grain_c4 --cipher grain --workload c4 --steps 1000
-  run mickey_c4 --cipher mickey2 --workload c4 --steps 300
-done
+D=gpurun_out/lp; mkdir -p $D
+timeout 900 python -m pytest tests/test_gpu_api.py tests/test_gpu_rowmajor_items.py tests/test_gpu_lfsr.py tests/test_gpu_random.py tests/test_gpu_fullsize.py -x -q -m gpu > $D/pytest.txt 2>&1
+tail -3 $D/pytest.txt
+run() { n=$1; shift; timeout 300 python bench.py --no-context --no-cpu-baseline --no-e2e --no-other-mode "$@" > $D/$n.json 2>$D/$n.err; }
+run lfsr_c2 --cipher lfsr128 --mode materialise --steps 20 --warmup 5
+run lfsr_c4 --cipher lfsr128 --mode materialise --workload c4 --steps 2000 --warmup 20
+run grain_c4 --cipher grain --mode materialise --workload c4 --steps 2000 --warmup 20
+for f in $D/*.json; do echo $f; python -c "import json,sys; d=json.load(open('$f')); print(d['value'], d['ms_per_step'], d['roofline']['frac'], d['clocks']['sm_mhz'])"; done
