@@ -97,10 +97,19 @@ int launch_aes(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st, uint64_t r
         occ_max = 1;
     occ = std::min(occ, occ_max);
     const uint64_t slots = uint64_t(h->num_sms) * occ * 4;
+    // Items (segment, warp-unit) are independent, so the split only trades
+    // the queue's tail against per-item overhead (state load, counter setup,
+    // checksum fold).  With at least two warp-units per slot: ~100 items per
+    // slot but no item shorter than 8 blocks (C2 4.29 vs 4.24 Tb/s at 32
+    // items per slot; 1024-bit rekey calls 3.81 vs 3.73 as whole units);
+    // fewer units than that (the paper shape) need the finer split for
+    // parallelism (C4: 2-block items 3.69, 8-block 3.64 Tb/s).
+    const bool many = h->units >= 2 * slots;
     const uint64_t quantum = bits >= 256 ? 256 : 128;
+    const uint64_t min_seg = many && bits >= 1024 && !h->opt_seg_clocks ? 1024 : quantum;
     uint64_t nseg = h->opt_seg_clocks ? (bits + h->opt_seg_clocks - 1) / h->opt_seg_clocks
-                                      : (32 * slots + h->units - 1) / h->units;
-    nseg = std::max<uint64_t>(1, std::min<uint64_t>(nseg, bits / quantum));
+                                      : ((many ? 100 : 32) * slots + h->units - 1) / h->units;
+    nseg = std::max<uint64_t>(1, std::min<uint64_t>(nseg, bits / min_seg));
     nseg = std::max<uint64_t>(nseg, (bits + MAX_SEG_CLOCKS - 1) / MAX_SEG_CLOCKS);
     const uint64_t seg = ((bits + nseg - 1) / nseg + quantum - 1) / quantum * quantum;
     a.nseg = (bits + seg - 1) / seg;
