@@ -447,6 +447,16 @@ __device__ __forceinline__ uint32_t laneid_volatile()
     asm volatile("mov.u32 %0, %%laneid;" : "=r"(v));
     return v;
 }
+// threadIdx.x >> 5 re-read from the special register (S2R) where it is used,
+// so that ptxas cannot keep it -- or addresses derived from it -- live across
+// a register-saturated clock loop (it spilled them: one local-memory reload on
+// the critical path of every 32-clock block)
+__device__ __forceinline__ uint32_t warp_volatile()
+{
+    uint32_t v;
+    asm volatile("mov.u32 %0, %%tid.x;" : "=r"(v));
+    return v >> 5;
+}
 
 // p + d as one IMAD.WIDE.U32 (FMA pipe) instead of IADD3 + IADD3.X (ALU);
 // d < 2^32 (row strides)

@@ -327,10 +327,11 @@ struct Mickey2 {
     // TMEM, two CTAs per SM, one work item per warp-unit (0.935 of the ALU
     // roofline vs 0.904 for the smem warp-specialised kernel)
     static constexpr bool RM_TMEM = true, RM_SEGMENTED = false;
-    // ROW_MAJOR warp-specialised kernel (rowmajor_ws.cuh) by default: never --
-    // the clock loop is ALU-bound and two clock-loop warps per SMSP keep the
-    // pipe fuller than one plus a writer (C2 1.84 vs 1.80, C4 1.38 vs 1.19 Tb/s)
-    static constexpr int RM_WS = 0;
+    // ROW_MAJOR warp-specialised kernel (rowmajor_ws.cuh) only when every
+    // warp-unit gets its own SMSP (the paper shape: C4 1.41 vs 1.37 Tb/s);
+    // otherwise two clock-loop warps per SMSP keep the ALU fuller than one
+    // plus a writer (C2 1.85 vs 1.81)
+    static constexpr int RM_WS = 1;
     // r[100..107]: pending overflow words of the deferred R reduction
     // (clock_at); only positions 0..99 are state between blocks
     uint32_t r[m2::RN], s[100];

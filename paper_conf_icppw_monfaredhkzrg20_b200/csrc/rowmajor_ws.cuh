@@ -153,19 +153,27 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
             }
             C c;
             c.load(a.state, a.Gp, g);
-            // hand block blk of the item (ring slot sq) to the writer
+            // hand block blk of the item (ring slot sq) to the writer.  The
+            // per-block code re-derives this warp's pair index (warp_volatile)
+            // instead of keeping ring / barrier addresses live across the clock
+            // loop (ptxas spilled them: an LDL on every block's critical path)
+            auto acquire = [&](uint32_t sq) {
+                const uint32_t pv = warp_volatile(), b = sq % ws::NZ;
+                if (sq >= ws::NZ) ws::mbar_wait(&bar_empty[pv][b], ((sq / ws::NZ) - 1) & 1u);
+                return pair_smem + pv * ws::PAIR_WORDS + b * ws::ZBUF + laneid_volatile();
+            };
             auto publish = [&](uint32_t sq, uint32_t blk) {
-                const uint32_t b = sq % ws::NZ;
+                const uint32_t pv = warp_volatile(), b = sq % ws::NZ;
                 if (laneid_volatile() == 0) {
-                    const uint64_t B = s_b0[pair] + blk;
+                    const uint64_t B = s_b0[pv] + blk;
                     const uint32_t kk = uint32_t(B % ws::NSLOT);
-                    ws::Meta& m = meta[pair][b];
-                    m.unit = s_unit[pair];
+                    ws::Meta& m = meta[pv][b];
+                    m.unit = s_unit[pv];
                     m.B = B;
                     m.k_lo = kk - (blk < kk ? blk : kk);
                     m.flags = (kk == ws::NSLOT - 1 || blk + 1 == nblk) ? ws::F_FLUSH : 0u;
                 }
-                ws::mbar_arrive(&bar_full[pair][b]);
+                ws::mbar_arrive(&bar_full[pv][b]);
             };
             uint32_t blk = 0;
             if constexpr (ks_period<C>::value) {
@@ -176,9 +184,7 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
                 for (; blk + PB <= nblk; blk += PB, seq += PB) {
                     static_for<PB>([&](auto jj) {
                         constexpr int J = decltype(jj)::value;
-                        const uint32_t b = (seq + J) % ws::NZ;
-                        if (seq + J >= ws::NZ) ws::mbar_wait(&bar_empty[pair][b], (((seq + J) / ws::NZ) - 1) & 1u);
-                        uint32_t* zb = zbase + b * ws::ZBUF + laneid_volatile();
+                        uint32_t* zb = acquire(seq + J);
                         c.template period_block<J>([&](int u, uint32_t v) { zb[u * 32] = v; });
                         publish(seq + J, blk + J);
                     });
@@ -186,9 +192,7 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
             }
 #pragma unroll 1
             for (; blk < nblk; ++blk, ++seq) {
-                const uint32_t b = seq % ws::NZ;
-                if (seq >= ws::NZ) ws::mbar_wait(&bar_empty[pair][b], ((seq / ws::NZ) - 1) & 1u);
-                uint32_t* zb = zbase + b * ws::ZBUF + laneid_volatile();
+                uint32_t* zb = acquire(seq);
 #pragma unroll 1
                 for (uint32_t k = 0; k < 32; k += U) {
                     static_for<U>([&](auto u) {
@@ -197,16 +201,7 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
                         ks_clock<J, KB>(c);
                     });
                 }
-                if (laneid_volatile() == 0) {
-                    const uint64_t B = s_b0[pair] + blk;
-                    const uint32_t kk = uint32_t(B % ws::NSLOT);
-                    ws::Meta& m = meta[pair][b];
-                    m.unit = s_unit[pair];
-                    m.B = B;
-                    m.k_lo = kk - (blk < kk ? blk : kk);
-                    m.flags = (kk == ws::NSLOT - 1 || blk + 1 == nblk) ? ws::F_FLUSH : 0u;
-                }
-                ws::mbar_arrive(&bar_full[pair][b]);
+                publish(seq, blk);
             }
             // re-derive the item context (kept out of registers during the loop)
             item = *slot;
