@@ -193,12 +193,14 @@ int64_t bsrng_copy_state(const bsrng_t* h, uint32_t* host_out, uint64_t words);
  *   "rm_ws"      : ROW_MAJOR kernel: -1 auto, 1 warp-specialised (a clock-loop
  *                  warp and a writer warp per SMSP; the writer transposes into
  *                  tensor memory and flushes 64 B per row; auto for the LFSR,
- *                  and for Grain when every warp-unit gets its own SMSP; AES:
+ *                  and for MICKEY and Grain when every warp-unit gets its
+ *                  own SMSP, unless rm_tmem / rm_wide are set; AES:
  *                  the block-lane kernel), 0 plain
  *   "rm_tmem"    : ROW_MAJOR plain kernel: stage the row segments in tensor
  *                  memory (TMEM, 256 columns per CTA, two CTAs per SM) (1)
  *                  or in shared memory (0); -1 = cipher default (MICKEY /
- *                  Grain 1, LFSR 0)
+ *                  Grain 1, LFSR 0).  Setting it (or
+ *                  rm_wide = 1) selects the plain kernel unless rm_ws is set
  *   "rm_tma"     : TMEM staging: whole-sector flushes of warps whose rows are
  *                  all real as TMA tensor stores when the row stride is a
  *                  multiple of 16 B (1, default) or as 8 B stores (0)

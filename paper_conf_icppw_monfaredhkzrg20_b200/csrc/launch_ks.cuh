@@ -45,7 +45,11 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
     // auto (C::RM_WS): 0 never, 1 when every warp-unit gets its own SMSP
     // (lone clock-loop warps), 2 always
     const bool lone = h->units <= uint64_t(h->num_sms) * 4;
-    const bool ws_pref = h->opt_rm_ws < 0 ? (C::RM_WS == 2 || (C::RM_WS == 1 && lone)) : (h->opt_rm_ws != 0);
+    // (an explicit plain-kernel staging choice -- rm_wide, rm_tmem -- turns the
+    // automatic writer-warp choice off)
+    const bool plain_asked = h->opt_rm_wide > 0 || h->opt_rm_tmem >= 0;
+    const bool ws_pref = h->opt_rm_ws < 0 ? (!plain_asked && (C::RM_WS == 2 || (C::RM_WS == 1 && lone)))
+                                          : (h->opt_rm_ws != 0);
     // calls longer than MAX_SEG_CLOCKS need time segments, i.e. the persistent queue
     const bool persistent = h->opt_sched != 0 || bits > MAX_SEG_CLOCKS;
     const bool ws = RM && ws_pref && persistent;

@@ -53,16 +53,19 @@ def test_zero_bits_is_noop(cipher):
 @pytest.mark.parametrize("cipher,opts", [
     ("mickey2", {"unroll": 4}), ("mickey2", {"sched": 0}),
     ("mickey2", {"ctas_per_sm": 2}), ("mickey2", {"rm_ws": 0}), ("mickey2", {"rm_ws": 1, "seg_clocks": 512}),
-    ("mickey2", {"rm_ws": 1}), ("mickey2", {"rm_tmem": 0}), ("mickey2", {"rm_tmem": 1, "seg_clocks": 384}),
+    ("mickey2", {"rm_ws": 1}), ("mickey2", {"rm_ws": 0, "rm_tmem": 0}),
+    ("mickey2", {"rm_ws": 0, "rm_tmem": 1, "seg_clocks": 384}),
     ("grain", {"unroll": 16}), ("grain", {"rm_ws": 1}), ("grain", {"sched": 0}),
-    ("grain", {"ctas_per_sm": 1, "seg_clocks": 256}),
-    ("grain", {"rm_tmem": 0}), ("grain", {"rm_tmem": 0, "unroll": 16}),
-    ("grain", {"rm_tmem": 0, "ctas_per_sm": 2, "seg_clocks": 384}),
+    ("grain", {"ctas_per_sm": 1, "seg_clocks": 256}), ("grain", {"rm_ws": 0, "ctas_per_sm": 1, "seg_clocks": 256}),
+    ("grain", {"rm_ws": 0, "rm_tmem": 0}), ("grain", {"rm_ws": 0, "rm_tmem": 0, "unroll": 16}),
+    ("grain", {"rm_ws": 0, "rm_tmem": 0, "ctas_per_sm": 2, "seg_clocks": 384}),
     ("mickey2", {"rm_ws": 0, "rm_tmem": 0}), ("mickey2", {"rm_ws": 0, "rm_tmem": 0, "seg_clocks": 160}),
     ("aes128ctr", {"ctas_per_sm": 1}), ("aes128ctr", {"rm_ws": 0}), ("aes128ctr", {"seg_clocks": 4096}),
     ("lfsr128", {}), ("lfsr128", {"rm_ws": 1, "seg_clocks": 512}), ("lfsr128", {"seg_clocks": 1536}),
 ])
 def test_options_stay_bit_exact(cipher, opts):
+    # 41 warp-units: MICKEY / Grain ROW_MAJOR default to the writer-warp kernel
+    # here, rm_ws = 0 selects the plain kernel
     n, bits = 32 * 40 + 9, 8192
     keys, ivs = inputs.make_inputs(cipher, n)
     want = _want(cipher, keys, ivs, bits)
@@ -135,26 +138,26 @@ def test_mickey_2_40_limit_boundary():
 
 
 @pytest.mark.parametrize("cipher,opts,bits", [
-    ("grain", {"rm_tmem": 1}, 8192),
-    ("grain", {"rm_tmem": 1}, 4416),                      # 552 B rows: 8 B-aligned flushes
-    ("grain", {"rm_tmem": 1, "seg_clocks": 160}, 2080),   # partial slots at segment ends
-    ("grain", {"rm_tmem": 1, "unroll": 16}, 4128),
-    ("grain", {"rm_tmem": 1, "sched": 0}, 2048),
-    ("grain", {"rm_tmem": 1, "ctas_per_sm": 2, "seg_clocks": 512}, 4096),
+    ("grain", {"rm_ws": 0, "rm_tmem": 1}, 8192),
+    ("grain", {"rm_ws": 0, "rm_tmem": 1}, 4416),                      # 552 B rows: 8 B-aligned flushes
+    ("grain", {"rm_ws": 0, "rm_tmem": 1, "seg_clocks": 160}, 2080),   # partial slots at segment ends
+    ("grain", {"rm_ws": 0, "rm_tmem": 1, "unroll": 16}, 4128),
+    ("grain", {"rm_ws": 0, "rm_tmem": 1, "sched": 0}, 2048),
+    ("grain", {"rm_ws": 0, "rm_tmem": 1, "ctas_per_sm": 2, "seg_clocks": 512}, 4096),
     ("mickey2", {"rm_ws": 0, "rm_tmem": 1}, 4416),
     ("mickey2", {"rm_ws": 0, "rm_tmem": 1, "seg_clocks": 96}, 1024),
-    ("grain", {"rm_tmem": 1, "rm_tma": 0}, 8192),        # 8 B global-store flush instead of TMA
+    ("grain", {"rm_ws": 0, "rm_tmem": 1, "rm_tma": 0}, 8192),        # 8 B global-store flush instead of TMA
     ("mickey2", {"rm_ws": 0, "rm_tmem": 1}, 8192),        # TMA flush (1 KB rows) for warp 0, 8 B for warp 1
-    ("grain", {"rm_tmem": 1, "rm_tma": 0}, 4416 + 256),  # double-buffered staging, progressive flush
+    ("grain", {"rm_ws": 0, "rm_tmem": 1, "rm_tma": 0}, 4416 + 256),  # double-buffered staging, progressive flush
     ("mickey2", {"rm_ws": 0, "rm_tmem": 1, "rm_tma": 0}, 2048 + 96),  # ... item ends mid-period
-    ("grain", {"rm_tmem": 1, "rm_dbl": 0}, 4416),          # single buffer
-    ("grain", {"rm_wide": 1}, 8192),                      # 64 B staging, whole 512-clock flushes
-    ("grain", {"rm_wide": 1}, 4416),                      # 552 B rows: word-by-word flushes
-    ("grain", {"rm_wide": 1, "seg_clocks": 160}, 2080),   # partial periods at segment ends
-    ("mickey2", {"rm_wide": 1}, 1024 + 512 + 96),
-    ("grain", {"rm_wide": 1, "unroll": 16, "seg_clocks": 1024}, 4096),
-    ("grain", {"rm_l2last": 0}, 8192),                     # evict-first TMA flush
-    ("grain", {"rm_l2last": 0, "rm_tma": 0}, 8192),        # evict-first 8 B sector flush
+    ("grain", {"rm_ws": 0, "rm_tmem": 1, "rm_dbl": 0}, 4416),          # single buffer
+    ("grain", {"rm_ws": 0, "rm_wide": 1}, 8192),                      # 64 B staging, whole 512-clock flushes
+    ("grain", {"rm_ws": 0, "rm_wide": 1}, 4416),                      # 552 B rows: word-by-word flushes
+    ("grain", {"rm_ws": 0, "rm_wide": 1, "seg_clocks": 160}, 2080),   # partial periods at segment ends
+    ("mickey2", {"rm_ws": 0, "rm_wide": 1}, 1024 + 512 + 96),
+    ("grain", {"rm_ws": 0, "rm_wide": 1, "unroll": 16, "seg_clocks": 1024}, 4096),
+    ("grain", {"rm_ws": 0, "rm_l2last": 0}, 8192),                     # evict-first TMA flush
+    ("grain", {"rm_ws": 0, "rm_l2last": 0, "rm_tma": 0}, 8192),        # evict-first 8 B sector flush
     ("grain", {"rm_ws": 1}, 4416),                         # writer warp, 552 B rows (STG.64 pieces)
     ("grain", {"rm_ws": 1, "seg_clocks": 512}, 4096 + 1024),
     ("mickey2", {"rm_ws": 1}, 4416),
@@ -166,7 +169,10 @@ def test_mickey_2_40_limit_boundary():
 ])
 def test_rm_tmem_staging_bit_exact(cipher, opts, bits):
     """ROW_MAJOR with the row segments staged in tensor memory (TMEM) instead
-    of shared memory: every flush path (16 B, 8 B, partial words) bit-exact."""
+    of shared memory: every flush path (16 B, 8 B, partial words) bit-exact.
+    n = 1289 is 41 warp-units, fewer than the SMSPs, where MICKEY and Grain
+    default to the writer-warp kernel; rm_ws = 0 selects the plain kernel's
+    staging variants."""
     n = 32 * 40 + 9
     keys, ivs = inputs.make_inputs(cipher, n)
     want = _want(cipher, keys, ivs, bits)
@@ -234,12 +240,15 @@ def test_device_input_rekey(cipher, n, misalign):
 
 
 @pytest.mark.parametrize("cipher,bits,opts", [
-    ("grain", 4096, {}), ("grain", 2048, {"seg_clocks": 512}), ("mickey2", 2048, {}), ("grain", 4096, {"rm_tma": 0}),
+    ("grain", 4096, {"rm_ws": 0}), ("grain", 2048, {"rm_ws": 0, "seg_clocks": 512}), ("mickey2", 2048, {"rm_ws": 0}),
+    ("grain", 4096, {"rm_ws": 0, "rm_tma": 0}),
 ])
 def test_rm_tma_flush_many_warps(cipher, bits, opts):
     """TMA tensor-store flushes (3-D view [q][group][byte] of the row-major
     output) from several warp-units at once plus a ragged tail unit that
-    falls back to global stores: every row bit-exact."""
+    falls back to global stores: every row bit-exact.  (129 warp-units, fewer
+    than the SMSPs: rm_ws = 0 keeps the plain kernel instead of the writer-warp
+    default.)"""
     n = 32 * 32 * 4 + 17
     keys, ivs = inputs.make_inputs(cipher, n)
     want = _want(cipher, keys, ivs, bits)

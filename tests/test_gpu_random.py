@@ -15,12 +15,16 @@ pytestmark = pytest.mark.gpu
 
 from paper_conf_icppw_monfaredhkzrg20_b200 import bsrng, inputs  # noqa: E402
 
+# n <= 7681 here is at most 241 warp-units, fewer than the SMSPs: MICKEY and
+# Grain ROW_MAJOR default to the writer-warp kernel, rm_ws = 0 reaches the
+# plain kernel's staging variants
+W = {"rm_ws": 0}
 OPTS = {
-    "mickey2": [{}, {"sched": 0}, {"rm_tmem": 0}, {"rm_ws": 1}, {"rm_tma": 0}, {"rm_wide": 1}, {"seg_clocks": 96},
-                {"ctas_per_sm": 1}, {"rm_l2last": 0}],
-    "grain": [{}, {"sched": 0}, {"rm_tmem": 0}, {"rm_ws": 1}, {"rm_ws": 0}, {"rm_tma": 0}, {"rm_wide": 1},
-              {"unroll": 16}, {"seg_clocks": 160}, {"ctas_per_sm": 1}, {"rm_dbl": 0}],
-    "lfsr128": [{}, {"sched": 0}, {"rm_ws": 0}, {"rm_ws": 1}, {"rm_wide": 1}, {"unroll": 16}, {"seg_clocks": 64}],
+    "mickey2": [{}, {"sched": 0}, {**W, "rm_tmem": 0}, W, {**W, "rm_tma": 0}, {**W, "rm_wide": 1},
+                {"seg_clocks": 96}, {**W, "ctas_per_sm": 1}, {**W, "rm_l2last": 0}],
+    "grain": [{}, {"sched": 0}, {**W, "rm_tmem": 0}, {"rm_ws": 1}, W, {**W, "rm_tma": 0}, {**W, "rm_wide": 1},
+              {"unroll": 16}, {"seg_clocks": 160}, {"ctas_per_sm": 1}, {**W, "rm_dbl": 0}],
+    "lfsr128": [{}, {"sched": 0}, {"rm_ws": 0}, {"rm_ws": 1}, {**W, "rm_wide": 1}, {"unroll": 16}, {"seg_clocks": 64}],
     "aes128ctr": [{}, {"rm_ws": 0}, {"ctas_per_sm": 1}, {"seg_clocks": 256}],
 }
 

@@ -84,7 +84,7 @@ _FORCED = [
     ("mickey2", {"ctas_per_sm": 1, "seg_clocks": 256, "rm_tmem": 0, "rm_ws": 0}, 1024),  # smem staging
     ("mickey2", {"seg_clocks": 256, "rm_ws": 1}, 1024),                        # warp-specialised
     ("grain", {"rm_wide": 1, "seg_clocks": 1024}, 2048),                      # 64 B staging, lone warps
-    ("lfsr128", {"rm_wide": 1, "seg_clocks": 512}, 2048),                     # 64 B staging
+    ("lfsr128", {"rm_ws": 0, "rm_wide": 1, "seg_clocks": 512}, 2048),         # 64 B staging
     ("lfsr128", {"ctas_per_sm": 1, "seg_clocks": 256}, 2048),                 # LFSR default (writer warp)
     ("lfsr128", {"seg_clocks": 512}, 2048 + 96),                              # period bodies + remainder
 ]

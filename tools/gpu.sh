@@ -78,9 +78,14 @@ captures)
   SKIP=0 capture preclock m2_init --layout checksum --bits 32 --reps 1
   SKIP=0 capture grain_init grain_init --cipher grain --layout checksum --bits 32 --reps 1 ;;
 sanitize)
-  for tool in memcheck racecheck synccheck; do
+  for tool in memcheck racecheck; do
     timeout 1500 compute-sanitizer --tool $tool --print-limit 20 python tools/sanitize_driver.py > $D/$tool.txt 2>&1
     echo "exit $?" >> $D/$tool.txt
+  done
+  for v in WS_ONLY NO_TMEM; do
+    env SANITIZE_$v=1 timeout 1500 compute-sanitizer --tool synccheck --print-limit 20 \
+      python tools/sanitize_driver.py > $D/synccheck_$v.txt 2>&1
+    echo "exit $?" >> $D/synccheck_$v.txt
   done ;;
 micro)
   (cd tools/microbench && ./alu_peak 200000 && ./curand_bench 4294967296 && ./write_peak) > $D/micro.log 2>&1 ;;
