@@ -509,6 +509,24 @@ __device__ __forceinline__ void tmem_ld16x256b_x4(uint32_t taddr, uint32_t (&v)[
         : "memory");
 }
 
+// The same for 8 repeats (64 columns, 32 registers): two row pairs per
+// tcgen05.wait::ld, so the flush loops pay the TMEM load latency once per four
+// rows instead of once per two (ncu: the writer warp's flush loop waited on
+// the x4 load's scoreboard for ~60% of its samples).
+__device__ __forceinline__ void tmem_ld16x256b_x8(uint32_t taddr, uint32_t (&v)[32])
+{
+    asm volatile(
+        "tcgen05.ld.sync.aligned.16x256b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, "
+        "%15, %16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, %29, %30, %31}, [%32];\n\t"
+        "tcgen05.wait::ld.sync.aligned;"
+        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+          "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15]),
+          "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]), "=r"(v[22]), "=r"(v[23]),
+          "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]), "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
+        : "r"(taddr)
+        : "memory");
+}
+
 // Whole-sector flush (slots 0..7 of every row, 8 B aligned rows) read back
 // with the 16x256b shape: four consecutive threads receive one TMEM lane's
 // (= one instance row's) 32 B sector, so each 8 B store instruction writes 8
@@ -655,42 +673,76 @@ __device__ __forceinline__ void rowmajor_store_tmem_wide(uint32_t tm, uint8_t* c
         const uint32_t na = nvalids[la], nb = nvalids[lb];
         if (a16 && __all_sync(0xFFFFFFFFu, (na & nb) == 32)) {
 #pragma unroll 1
-            for (uint32_t q = 0; q < 32; q += 2) {
-                uint32_t v[16];  // rows q (v0..7) and q+1 (v8..15) of lanes la (v[4i], v[4i+1]) / lb
-                tmem_ld16x256b_x4(tm + ((16 * h) << 16) + q * 16, v);
-                st128_hint(pa, v[0], v[1], v[4], v[5], pol);
-                st128_hint(pb, v[2], v[3], v[6], v[7], pol);
-                pa = add_fma(pa, row_bytes);
-                pb = add_fma(pb, row_bytes);
-                st128_hint(pa, v[8], v[9], v[12], v[13], pol);
-                st128_hint(pb, v[10], v[11], v[14], v[15], pol);
-                pa = add_fma(pa, row_bytes);
-                pb = add_fma(pb, row_bytes);
+            for (uint32_t q = 0; q < 32; q += 4) {
+                uint32_t v[32];  // rows q..q+3 (v[8r..8r+7]) of lanes la (v[8r+4i], +1) / lb (+2, +3)
+                tmem_ld16x256b_x8(tm + ((16 * h) << 16) + q * 16, v);
+#pragma unroll
+                for (int r = 0; r < 4; ++r) {
+                    st128_hint(pa, v[8 * r], v[8 * r + 1], v[8 * r + 4], v[8 * r + 5], pol);
+                    st128_hint(pb, v[8 * r + 2], v[8 * r + 3], v[8 * r + 6], v[8 * r + 7], pol);
+                    pa = add_fma(pa, row_bytes);
+                    pb = add_fma(pb, row_bytes);
+                }
             }
             continue;
         }
 #pragma unroll 1
-        for (uint32_t q = 0; q < 32; q += 2) {
-            uint32_t v[16];
-            tmem_ld16x256b_x4(tm + ((16 * h) << 16) + q * 16, v);
-            if (q < na) st_piece16(pa, v[0], v[1], v[4], v[5], pol, a16);
-            if (q < nb) st_piece16(pb, v[2], v[3], v[6], v[7], pol, a16);
-            pa += row_bytes;
-            pb += row_bytes;
-            if (q + 1 < na) st_piece16(pa, v[8], v[9], v[12], v[13], pol, a16);
-            if (q + 1 < nb) st_piece16(pb, v[10], v[11], v[14], v[15], pol, a16);
-            pa += row_bytes;
-            pb += row_bytes;
+        for (uint32_t q = 0; q < 32; q += 4) {
+            uint32_t v[32];
+            tmem_ld16x256b_x8(tm + ((16 * h) << 16) + q * 16, v);
+#pragma unroll
+            for (int r = 0; r < 4; ++r) {
+                if (q + r < na) st_piece16(pa, v[8 * r], v[8 * r + 1], v[8 * r + 4], v[8 * r + 5], pol, a16);
+                if (q + r < nb) st_piece16(pb, v[8 * r + 2], v[8 * r + 3], v[8 * r + 6], v[8 * r + 7], pol, a16);
+                pa += row_bytes;
+                pb += row_bytes;
+            }
         }
+    }
+}
+
+__device__ __forceinline__ void st32_hint(uint8_t* p, uint32_t a, uint64_t pol)
+{
+    asm volatile("st.global.L2::cache_hint.u32 [%0], %1, %2;" ::"l"(p), "r"(a), "l"(pol) : "memory");
+}
+// Store the run of slots [m0, m1] (0 <= m0, m1 <= 3; empty if m0 > m1) of one
+// row's 16 B piece w[0..3]; A = the address slot 0 of the piece would have.
+// Widest aligned stores: 16 B for a whole 16 B aligned piece, else 8 B pairs
+// on 8 B boundaries and 4 B singles (rows are at least 4 B aligned).
+__device__ __forceinline__ void st_run4(uint8_t* A, uint32_t w0, uint32_t w1, uint32_t w2, uint32_t w3, int m0,
+                                        int m1, uint64_t pol)
+{
+    const bool r0 = m0 <= 0 && 0 <= m1, r1 = m0 <= 1 && 1 <= m1, r2 = m0 <= 2 && 2 <= m1, r3 = m0 <= 3 && 3 <= m1;
+    const uint32_t al = uint32_t(reinterpret_cast<uintptr_t>(A)) & 15u;
+    if ((al & 7u) == 0) {
+        if (r0 && r3 && al == 0) {
+            st128_hint(A, w0, w1, w2, w3, pol);
+            return;
+        }
+        if (r0 && r1) st64_hint(A, w0, w1, pol);
+        else if (r0) st32_hint(A, w0, pol);
+        else if (r1) st32_hint(A + 4, w1, pol);
+        if (r2 && r3) st64_hint(A + 8, w2, w3, pol);
+        else if (r2) st32_hint(A + 8, w2, pol);
+        else if (r3) st32_hint(A + 12, w3, pol);
+    } else {
+        if (r0) st32_hint(A, w0, pol);
+        if (r1 && r2 && (al & 7u) == 4u) st64_hint(A + 4, w1, w2, pol);
+        else {
+            if (r1) st32_hint(A + 4, w1, pol);
+            if (r2) st32_hint(A + 8, w2, pol);
+        }
+        if (r3) st32_hint(A + 12, w3, pol);
     }
 }
 
 // Partial 64 B flush: slots [k_lo, k_hi] only (item boundaries that are not
 // whole 512-clock periods, e.g. the paper shape's 4416 clocks = 8 periods + 10
-// slots; rows that are only 4 B aligned).  Same 16x256b read-back as the
-// whole flush, one predicated 4 B store per slot: each store instruction
-// covers 8 rows x 4 slots, instead of 32 rows x 1 slot from each thread's own
-// rows (the first version wrote the paper shape's last 10 slots that way).
+// slots).  Same 16x256b read-back as the whole flush; thread j = t%4 holds
+// slots 4j..4j+3 of its rows and stores the part of them inside [k_lo, k_hi]
+// with the widest aligned stores (st_run4): the paper shape's closing 40 B
+// leave as 8 B stores instead of one 4 B store per slot (this flush runs after
+// the clock loop has ended, so it is the kernel's tail).
 __device__ __forceinline__ void rowmajor_store_tmem_wide_partial(uint32_t tm, uint8_t* const* row0s,
                                                                  const uint32_t* nvalids, uint64_t row_bytes,
                                                                  uint32_t k_lo, uint32_t k_hi, uint64_t col)
@@ -698,28 +750,29 @@ __device__ __forceinline__ void rowmajor_store_tmem_wide_partial(uint32_t tm, ui
     tmem_wait_st();
     const uint32_t t = laneid_volatile();
     const uint32_t j = t & 3u;
+    const uint64_t pol = l2_evict_last_policy();
+    // this thread's run [m0, m1] of slots 4j + m inside [k_lo, k_hi]
+    const int lo = int(k_lo > 4 * j ? k_lo : 4 * j), hi = int(k_hi < 4 * j + 3 ? k_hi : 4 * j + 3);
+    const int m0 = lo - int(4 * j), m1 = hi - int(4 * j);  // empty when lo > hi
+    // A = address of slot 4j: piece start + (4j - k_lo) words (may precede it)
+    const int64_t off = int64_t(col) + 4 * (int64_t(4 * j) - int64_t(k_lo));
 #pragma unroll 1
     for (uint32_t h = 0; h < 2; ++h) {
         const uint32_t la = 16 * h + (t >> 2), lb = la + 8;
-        uint8_t* pa = row0s[la] + col;
-        uint8_t* pb = row0s[lb] + col;
+        uint8_t* pa = row0s[la] + off;
+        uint8_t* pb = row0s[lb] + off;
         const uint32_t na = nvalids[la], nb = nvalids[lb];
 #pragma unroll 1
-        for (uint32_t q = 0; q < 32; q += 2) {
-            uint32_t v[16];
-            tmem_ld16x256b_x4(tm + ((16 * h) << 16) + q * 16, v);
+        for (uint32_t q = 0; q < 32; q += 4) {
+            uint32_t v[32];
+            tmem_ld16x256b_x8(tm + ((16 * h) << 16) + q * 16, v);
+            if (m0 <= m1) {
 #pragma unroll
-            for (int r = 0; r < 2; ++r) {
-#pragma unroll
-                for (int m = 0; m < 4; ++m) {
-                    // slot 4j + m sits in v[8r + (m & 1) + (m & 2 ? 4 : 0)] (lane la), +2 (lane lb)
-                    const int iv = 8 * r + (m & 1) + ((m & 2) ? 4 : 0);
-                    const uint32_t sl = 4 * j + m;
-                    if (sl >= k_lo && sl <= k_hi) {
-                        if (q + r < na) __stcs(reinterpret_cast<uint32_t*>(pa + (q + r) * row_bytes) + (sl - k_lo), v[iv]);
-                        if (q + r < nb)
-                            __stcs(reinterpret_cast<uint32_t*>(pb + (q + r) * row_bytes) + (sl - k_lo), v[iv + 2]);
-                    }
+                for (int r = 0; r < 4; ++r) {
+                    if (q + r < na) st_run4(pa, v[8 * r], v[8 * r + 1], v[8 * r + 4], v[8 * r + 5], m0, m1, pol);
+                    if (q + r < nb) st_run4(pb, v[8 * r + 2], v[8 * r + 3], v[8 * r + 6], v[8 * r + 7], m0, m1, pol);
+                    pa += row_bytes;
+                    pb += row_bytes;
                 }
             }
         }

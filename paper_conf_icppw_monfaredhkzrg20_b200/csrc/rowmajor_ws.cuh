@@ -33,9 +33,12 @@ namespace ws {
 constexpr int NCOMP = 4;                    // compute warps per CTA (one per SMSP)
 constexpr int BLOCK = 2 * NCOMP * 32;       // + one writer warp each
 constexpr int ZBUF = 32 * 32;               // words in one z block: [t][lane]
-constexpr int NZ = 4;                       // z blocks in flight per pair (absorb the flush bursts)
+#ifndef WS_NZ
+#define WS_NZ 4
+#endif
+constexpr int NZ = WS_NZ;                   // z blocks in flight per pair (absorb the flush bursts)
 constexpr int PAIR_WORDS = NZ * ZBUF;
-constexpr size_t SMEM_BYTES = size_t(NCOMP) * PAIR_WORDS * 4;  // 64 KB
+constexpr size_t SMEM_BYTES = size_t(NCOMP) * PAIR_WORDS * 4;  // 16 KB per z block
 constexpr uint32_t NSLOT = 16;              // 32-clock blocks per 64 B row piece
 #ifndef WRITER_SLEEP_NS
 #define WRITER_SLEEP_NS 200
