@@ -34,11 +34,16 @@ constexpr int NCOMP = 4;                    // compute warps per CTA (one per SM
 constexpr int BLOCK = 2 * NCOMP * 32;       // + one writer warp each
 constexpr int ZBUF = 32 * 32;               // words in one z block: [t][lane]
 #ifndef WS_NZ
-#define WS_NZ 4
+#define WS_NZ 8
 #endif
 constexpr int NZ = WS_NZ;                   // z blocks in flight per pair (absorb the flush bursts)
+#ifndef WS_G
+#define WS_G 4
+#endif
+constexpr int G = WS_G;                     // z blocks per empty-barrier wait of the clock-loop warp
+static_assert(G >= 1 && G <= NZ, "a wait group must fit in the ring");
 constexpr int PAIR_WORDS = NZ * ZBUF;
-constexpr size_t SMEM_BYTES = size_t(NCOMP) * PAIR_WORDS * 4;  // 16 KB per z block
+constexpr size_t SMEM_BYTES = size_t(NCOMP) * PAIR_WORDS * 4;  // 4 KB per z block: 128 KB
 constexpr uint32_t NSLOT = 16;              // 32-clock blocks per 64 B row piece
 #ifndef WRITER_SLEEP_NS
 #define WRITER_SLEEP_NS 200
@@ -160,10 +165,24 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
             // per-block code re-derives this warp's pair index (warp_volatile)
             // instead of keeping ring / barrier addresses live across the clock
             // loop (ptxas spilled them: an LDL on every block's critical path)
-            auto acquire = [&](uint32_t sq) {
+            // ring slot of z block sq (its empty barrier already waited for)
+            auto slot_ptr = [&](uint32_t sq) {
                 const uint32_t pv = warp_volatile(), b = sq % ws::NZ;
-                if (sq >= ws::NZ) ws::mbar_wait(&bar_empty[pv][b], ((sq / ws::NZ) - 1) & 1u);
                 return pair_smem + pv * ws::PAIR_WORDS + b * ws::ZBUF + laneid_volatile();
+            };
+            // The writer consumes z blocks in order, so slot sq's empty barrier
+            // having completed its phase implies the same for every earlier
+            // slot: one wait covers a group of WS_G blocks (the try_wait's
+            // round trip stalled the lone clock-loop warp once per block).
+            auto wait_empty = [&](uint32_t sq) {
+                if (sq >= ws::NZ) {
+                    const uint32_t pv = warp_volatile(), b = sq % ws::NZ;
+                    ws::mbar_wait(&bar_empty[pv][b], ((sq / ws::NZ) - 1) & 1u);
+                }
+            };
+            auto acquire = [&](uint32_t sq) {
+                wait_empty(sq);
+                return slot_ptr(sq);
             };
             auto publish = [&](uint32_t sq, uint32_t blk) {
                 const uint32_t pv = warp_volatile(), b = sq % ws::NZ;
@@ -194,17 +213,22 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
                 }
             }
 #pragma unroll 1
-            for (; blk < nblk; ++blk, ++seq) {
-                uint32_t* zb = acquire(seq);
+            while (blk < nblk) {
+                const uint32_t gn = nblk - blk < uint32_t(ws::G) ? nblk - blk : uint32_t(ws::G);
+                wait_empty(seq + gn - 1);
 #pragma unroll 1
-                for (uint32_t k = 0; k < 32; k += U) {
-                    static_for<U>([&](auto u) {
-                        constexpr int J = decltype(u)::value % KB;
-                        zb[(k + decltype(u)::value) * 32] = ks_z<J, KB>(c);
-                        ks_clock<J, KB>(c);
-                    });
+                for (uint32_t gi = 0; gi < gn; ++gi, ++blk, ++seq) {
+                    uint32_t* zb = slot_ptr(seq);
+#pragma unroll 1
+                    for (uint32_t k = 0; k < 32; k += U) {
+                        static_for<U>([&](auto u) {
+                            constexpr int J = decltype(u)::value % KB;
+                            zb[(k + decltype(u)::value) * 32] = ks_z<J, KB>(c);
+                            ks_clock<J, KB>(c);
+                        });
+                    }
+                    publish(seq, blk);
                 }
-                publish(seq, blk);
             }
             // re-derive the item context (kept out of registers during the loop)
             item = *slot;
@@ -237,9 +261,18 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
             const uint32_t k_lo = vm.k_lo;
             const uint32_t k = uint32_t(B % ws::NSLOT);
             const uint32_t tm = *reinterpret_cast<volatile uint32_t*>(&s_tmem) + (pair << 21);
+            // WS_EXPERIMENT_NO_WRITER (measurement builds only, wrong output):
+            // the writer skips its transposes and flushes, which isolates the
+            // lone clock-loop warp's own rate
+#ifndef WS_EXPERIMENT_NO_WRITER
             rowmajor_transpose_smem_tmem<C::MSB_FIRST, 16>(zbase + b * ws::ZBUF + lane, tm, wide_col(k));
+#endif
             ws::mbar_arrive(&bar_empty[pair][b]);
+#if defined(WS_EXPERIMENT_NO_WRITER) || defined(WS_EXPERIMENT_NO_FLUSH)
+            if (false) {
+#else
             if (flags & ws::F_FLUSH) {
+#endif
                 const uint64_t first = (unit * 32u + lane) * 32u;
                 const uint32_t nvalid = first >= a.n ? 0u : uint32_t(a.n - first < 32 ? a.n - first : 32);
                 uint8_t* row0 = static_cast<uint8_t*>(a.out) + (nvalid ? first : 0) * a.row_bytes;
