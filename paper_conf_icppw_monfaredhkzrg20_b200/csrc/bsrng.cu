@@ -447,7 +447,7 @@ int bsrng_set_option(bsrng_t* h, const char* key, int64_t value)
         if (!ok) return fail(BSRNG_EINVAL, "unroll must be %s", wide ? "16 or 32" : "4 (MICKEY; AES: none)");
         h->opt_unroll = int(value);
     } else if (!strcmp(key, "rm_ws")) {
-        if (value < -1 || value > 1) return fail(BSRNG_EINVAL, "rm_ws must be -1 (auto), 0 or 1");
+        if (value < -1 || value > 2) return fail(BSRNG_EINVAL, "rm_ws must be -1 (auto), 0, 1 or 2");
         h->opt_rm_ws = int(value);
     } else if (!strcmp(key, "rm_dbl")) {
         if (int rc = in01("rm_dbl")) return rc;

@@ -9,6 +9,7 @@
 //   ROW_MAJOR, TMEM + dbl : keystream_kernel<C, ROW_MAJOR, U, .., TMEM, DBL>
 //   ROW_MAJOR, TMEM 64 B  : keystream_kernel<C, ROW_MAJOR, U, .., TMEM, -, WIDE>
 //   ROW_MAJOR, specialised: keystream_rm_ws_kernel<C, U>   (compute + writer warps, TMEM 64 B staging)
+//   ROW_MAJOR, 2 writers  : keystream_rm_ws2_kernel<C, U>  (per clock-loop warp; 128 B per row per flush)
 #pragma once
 #include <algorithm>
 #include <cstdio>
@@ -17,6 +18,7 @@
 #include "internal.h"
 #include "keystream.cuh"
 #include "rowmajor_ws.cuh"
+#include "rowmajor_ws2.cuh"
 
 namespace bsrng_impl {
 
@@ -48,11 +50,14 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
     // (an explicit plain-kernel staging choice -- rm_wide, rm_tmem -- turns the
     // automatic writer-warp choice off)
     const bool plain_asked = h->opt_rm_wide > 0 || h->opt_rm_tmem >= 0;
-    const bool ws_pref = h->opt_rm_ws < 0 ? (!plain_asked && (C::RM_WS == 2 || (C::RM_WS == 1 && lone)))
-                                          : (h->opt_rm_ws != 0);
+    // 3: the two-writers-per-stream kernel (rowmajor_ws2.cuh, 128 B per row per flush)
+    const int ws_kind = h->opt_rm_ws < 0
+                            ? (plain_asked ? 0 : C::RM_WS == 3 ? 2 : (C::RM_WS == 2 || (C::RM_WS == 1 && lone)) ? 1 : 0)
+                            : h->opt_rm_ws;
     // calls longer than MAX_SEG_CLOCKS need time segments, i.e. the persistent queue
     const bool persistent = h->opt_sched != 0 || bits > MAX_SEG_CLOCKS;
-    const bool ws = RM && ws_pref && persistent;
+    const bool ws2 = RM && ws_kind == 2 && persistent;
+    const bool ws = RM && ws_kind != 0 && persistent;
     // 64 B TMEM staging (keystream.cuh wide_col): one clock-loop warp per
     // SMSP with all 512 columns, so each flush writes 64 B per row
     const bool wide = RM && !ws && h->opt_rm_wide > 0;
@@ -95,6 +100,19 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
         block = bsk::ws::BLOCK;
         compute_warps = bsk::ws::NCOMP;
         smem = bsk::ws::SMEM_BYTES;
+        // built for the output-bound ciphers only (C::RM_WS >= 2: the LFSR)
+        if constexpr (C::RM_WS >= 2) {
+            if (ws2) {
+                kern = &bsk::keystream_rm_ws2_kernel<C, C::U_DEFAULT>;
+                if (h->opt_unroll == C::U_ALT0) kern = &bsk::keystream_rm_ws2_kernel<C, C::U_ALT0>;
+                if (h->opt_unroll == C::U_ALT1) kern = &bsk::keystream_rm_ws2_kernel<C, C::U_ALT1>;
+                block = bsk::ws2::BLOCK;
+                compute_warps = bsk::ws2::NSTREAM;
+                smem = bsk::ws2::SMEM_BYTES;
+            }
+        } else if (ws2) {
+            return fail(BSRNG_EINVAL, "rm_ws = 2 is built for the LFSR only");
+        }
     }
     if (int rc = set_smem(reinterpret_cast<const void*>(kern), smem)) return rc;
     unsigned grid;
@@ -146,7 +164,7 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
         nseg = std::max<uint64_t>(nseg, (bits + MAX_SEG_CLOCKS - 1) / MAX_SEG_CLOCKS);
         // whole 256-clock blocks keep ROW_MAJOR sector flushes full (32 B/row;
         // 512 clocks = 64 B for the wide staging)
-        const uint64_t q_full = (wide || ws) ? 512 : 256;
+        const uint64_t q_full = ws2 ? 1024 : (wide || ws) ? 512 : 256;
         const uint64_t quantum = bits >= q_full ? q_full : 32;
         uint64_t seg = ((bits + nseg - 1) / nseg + quantum - 1) / quantum * quantum;
         nseg = (bits + seg - 1) / seg;

@@ -62,6 +62,8 @@ def test_zero_bits_is_noop(cipher):
     ("mickey2", {"rm_ws": 0, "rm_tmem": 0}), ("mickey2", {"rm_ws": 0, "rm_tmem": 0, "seg_clocks": 160}),
     ("aes128ctr", {"ctas_per_sm": 1}), ("aes128ctr", {"rm_ws": 0}), ("aes128ctr", {"seg_clocks": 4096}),
     ("lfsr128", {}), ("lfsr128", {"rm_ws": 1, "seg_clocks": 512}), ("lfsr128", {"seg_clocks": 1536}),
+    ("lfsr128", {"rm_ws": 2}), ("lfsr128", {"rm_ws": 2, "seg_clocks": 1024}), ("lfsr128", {"rm_ws": 2, "seg_clocks": 3072}),
+    ("lfsr128", {"rm_ws": 2, "unroll": 16, "seg_clocks": 2048}),
 ])
 def test_options_stay_bit_exact(cipher, opts):
     # 41 warp-units: MICKEY / Grain ROW_MAJOR default to the writer-warp kernel
@@ -86,7 +88,7 @@ def test_options_stay_bit_exact(cipher, opts):
 def test_option_validation():
     keys, ivs = inputs.make_inputs("grain", 32)
     g = bsrng.Generator("grain", keys, ivs)
-    for k, v in (("unroll", 4), ("unroll", 8), ("sched", 2), ("seg_clocks", 33), ("ctas_per_sm", 99), ("rm_ws", 5),
+    for k, v in (("unroll", 4), ("unroll", 8), ("sched", 2), ("seg_clocks", 33), ("ctas_per_sm", 99), ("rm_ws", 5), ("rm_ws", 3),
                  ("rm_slots", 4), ("rm_zreg", 0), ("rm_tmem", 2), ("rm_tma", 2), ("rm_dbl", 2), ("init_fused", 2)):
         with pytest.raises(bsrng.BsrngError) as e:
             g.set_option(k, v)

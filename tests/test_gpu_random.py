@@ -24,7 +24,8 @@ OPTS = {
                 {"seg_clocks": 96}, {**W, "ctas_per_sm": 1}, {**W, "rm_l2last": 0}],
     "grain": [{}, {"sched": 0}, {**W, "rm_tmem": 0}, {"rm_ws": 1}, W, {**W, "rm_tma": 0}, {**W, "rm_wide": 1},
               {"unroll": 16}, {"seg_clocks": 160}, {"ctas_per_sm": 1}, {**W, "rm_dbl": 0}],
-    "lfsr128": [{}, {"sched": 0}, {"rm_ws": 0}, {"rm_ws": 1}, {**W, "rm_wide": 1}, {"unroll": 16}, {"seg_clocks": 64}],
+    "lfsr128": [{}, {"sched": 0}, {"rm_ws": 0}, {"rm_ws": 1}, {"rm_ws": 2}, {"rm_ws": 2, "seg_clocks": 96}, {**W, "rm_wide": 1},
+                {"unroll": 16}, {"seg_clocks": 64}],
     "aes128ctr": [{}, {"rm_ws": 0}, {"ctas_per_sm": 1}, {"seg_clocks": 256}],
 }
 

@@ -87,6 +87,10 @@ _FORCED = [
     ("lfsr128", {"rm_ws": 0, "rm_wide": 1, "seg_clocks": 512}, 2048),         # 64 B staging
     ("lfsr128", {"ctas_per_sm": 1, "seg_clocks": 256}, 2048),                 # LFSR default (writer warp)
     ("lfsr128", {"seg_clocks": 512}, 2048 + 96),                              # period bodies + remainder
+    ("lfsr128", {"rm_ws": 2, "seg_clocks": 1024}, 4096),                      # two writers per stream, 128 B
+    ("lfsr128", {"rm_ws": 2}, 2048 + 256 + 96),                               # ragged last period: partial flushes
+    ("lfsr128", {"rm_ws": 2, "seg_clocks": 256}, 768),                        # items start mid-period (k_lo > 0)
+    ("lfsr128", {"rm_ws": 2, "seg_clocks": 160}, 480),                        # skip blocks at unaligned item starts
 ]
 
 

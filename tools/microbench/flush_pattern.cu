@@ -16,7 +16,13 @@
 #include <cstdint>
 #include <cstdio>
 
-enum { QUAD_G, QUAD_Q, PAIR_G, PAIR_Q, ONE, SEG64, SEG128, SEG256, MIX };
+enum { QUAD_G, QUAD_Q, PAIR_G, PAIR_Q, ONE, SEG64, SEG128, SEG256, MIX, SPLIT128, SEG64_2W };
+// SPLIT128: warps 2p, 2p+1 of a CTA share one unit of 1024 rows; every flush
+//   writes 128 B of each row, warp 2p the row's 32 B sectors 0 and 2, warp
+//   2p+1 sectors 1 and 3 (16x256b-style: 4 lanes x 16 B per row, 8 rows per
+//   STG.128) -- two writer warps in two TMEM lane quarters per stream
+// SEG64_2W: SEG64 with only 2 of the 4 warps of a CTA working (half the rows
+//   in flight per SM)
 // store cache policy: 0 = evict-first (st.global.cs), 1 = default (write-back,
 // L2 evict_normal), 2 = L2 evict_last (createpolicy)
 template <int POL>
@@ -53,6 +59,26 @@ template <int V, int POL>
 __global__ void __launch_bounds__(128) flush_kernel(uint8_t* out, uint64_t pitch, uint32_t units, uint32_t seed)
 {
     const uint32_t lane = threadIdx.x & 31;
+    if (V == SPLIT128 || V == SEG64_2W) {
+        const uint32_t wi = threadIdx.x >> 5;
+        if (V == SEG64_2W && (wi & 1)) return;
+        const uint32_t npairs = gridDim.x * 2;
+        const uint32_t half = wi & 1;
+        for (uint32_t w = blockIdx.x * 2 + (wi >> 1); w < units; w += npairs) {
+            uint8_t* base = out + uint64_t(w) * 1024 * pitch;
+            const uint32_t bpr = V == SPLIT128 ? 128 : 64;
+            for (uint64_t c = 0; c < pitch; c += bpr) {
+                const uint32_t v = seed ^ uint32_t(c) ^ w;
+#pragma unroll 4
+                for (uint32_t it = 0; it < 128; ++it) {
+                    const uint32_t row = it * 8 + (lane >> 2), j = lane & 3;
+                    const uint32_t off = V == SPLIT128 ? 32 * (2 * (j >> 1) + half) + 16 * (j & 1) : 16 * j;
+                    st128<POL>(base + uint64_t(row) * pitch + c + off, make_uint4(v, it, lane, 5));
+                }
+            }
+        }
+        return;
+    }
     const uint32_t nwarps = gridDim.x * 4;
     for (uint32_t w = blockIdx.x * 4 + (threadIdx.x >> 5); w < units; w += nwarps) {
         uint8_t* base = out + uint64_t(w) * 1024 * pitch;
@@ -174,6 +200,11 @@ int main()
             run<SEG128, 0>("seg128", buf, pitch, units, sms, ctas);
             run<SEG128, 2>("seg128", buf, pitch, units, sms, ctas);
             run<SEG256, 0>("seg256", buf, pitch, units, sms, ctas);
+            if (ctas == 1) {
+                run<SPLIT128, 2>("split128_2streams", buf, pitch, units, sms, ctas);
+                run<SPLIT128, 1>("split128_2streams", buf, pitch, units, sms, ctas);
+                run<SEG64_2W, 2>("seg64_2streams", buf, pitch, units, sms, ctas);
+            }
             if (ctas == 2) {
                 run<MIX, 0>("mix_64_32", buf, pitch, units, sms, ctas);
                 run<MIX, 2>("mix_64_32", buf, pitch, units, sms, ctas);
