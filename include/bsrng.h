@@ -192,12 +192,12 @@ int64_t bsrng_copy_state(const bsrng_t* h, uint32_t* host_out, uint64_t words);
  *                  MICKEY 4 (the only one built); 0 = default
  *   "rm_ws"      : ROW_MAJOR kernel: -1 auto, 1 warp-specialised (a clock-loop
  *                  warp and a writer warp per SMSP; the writer transposes into
- *                  tensor memory and flushes 64 B per row; auto for the LFSR,
- *                  and for MICKEY and Grain when every warp-unit gets its
- *                  own SMSP, unless rm_tmem / rm_wide are set; AES:
- *                  the block-lane kernel), 2 two writer warps per clock-loop
- *                  warp (two streams per SM, 128 B per row per flush, each
- *                  writer two 32 B sectors of it), 0 plain
+ *                  tensor memory and flushes 64 B per row; auto for MICKEY
+ *                  and Grain when every warp-unit gets its own SMSP, unless
+ *                  rm_tmem / rm_wide are set; AES: the block-lane kernel),
+ *                  2 two writer warps per clock-loop warp (two streams per
+ *                  SM, 128 B per row per flush, each writer two 32 B sectors
+ *                  of it; LFSR only, its auto choice), 0 plain
  *   "rm_tmem"    : ROW_MAJOR plain kernel: stage the row segments in tensor
  *                  memory (TMEM, 256 columns per CTA, two CTAs per SM) (1)
  *                  or in shared memory (0); -1 = cipher default (MICKEY /

@@ -22,11 +22,12 @@ struct Lfsr128 {
     static constexpr bool MSB_FIRST = true;
     static constexpr int U_DEFAULT = 32, U_ALT0 = 16, U_ALT1 = 16;
     static constexpr bool RM_TMEM = false, RM_SEGMENTED = true;
-    // ROW_MAJOR: always the warp-specialised kernel with 64 B TMEM staging per
-    // row (rowmajor_ws.cuh): 2 LOP3 per clock leave the output path as the
-    // whole cost, and 64 B per row per flush is what the DRAM needs (C2 26.4
-    // vs 11.9 Tb/s with 32 B smem staging)
-    static constexpr int RM_WS = 2;
+    // ROW_MAJOR: always a warp-specialised kernel (2 LOP3 per clock leave the
+    // output path as the whole cost): two writer warps per clock-loop warp,
+    // two streams per SM, 128 B row pieces written as sector pairs
+    // (rowmajor_ws2.cuh; C2 27.5 Tb/s), rather than one writer per stream with
+    // 64 B pieces (rowmajor_ws.cuh, 26.3; 11.9 with 32 B smem staging)
+    static constexpr int RM_WS = 3;
     // consume: one 128-clock body (the rotation period), no moves (keystream.cuh)
     static constexpr int U_CONSUME = 128;
     static constexpr bool CONSUME_PERIOD = true;
