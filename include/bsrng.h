@@ -214,6 +214,11 @@ int64_t bsrng_copy_state(const bsrng_t* h, uint32_t* host_out, uint64_t words);
  *                  clock-loop warp per SMSP (1) or not (0, default)
  *   "rm_l2last"  : ROW_MAJOR 32 B flushes (TMA / 8 B stores) with an L2
  *                  evict_last hint (1, default) or evict-first (0)
+ *   "rm_phase"   : writer-warp kernel (rm_ws = 1): stagger the warp-units'
+ *                  64 B flush periods by 0, 2, .., 14 blocks (unit mod 8) so
+ *                  that they do not all write at once (1), or flush every
+ *                  unit in the same block (0); -1 (default) = on when the row
+ *                  stride is not a multiple of 16 B (the paper's 552 B rows)
  *   "init_fused" : create/rekey: slicing fused into the initialisation kernel
  *                  (1, default) or the separate ballot slice (+ preclock)
  *                  kernels (0)

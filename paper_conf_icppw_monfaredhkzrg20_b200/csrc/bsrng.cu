@@ -461,6 +461,9 @@ int bsrng_set_option(bsrng_t* h, const char* key, int64_t value)
     } else if (!strcmp(key, "rm_l2last")) {
         if (int rc = in01("rm_l2last")) return rc;
         h->opt_rm_l2last = int(value);
+    } else if (!strcmp(key, "rm_phase")) {
+        if (value < -1 || value > 1) return fail(BSRNG_EINVAL, "rm_phase must be -1 (auto), 0 or 1");
+        h->opt_rm_phase = int(value);
     } else if (!strcmp(key, "rm_tmem")) {
         if (value < -1 || value > 1) return fail(BSRNG_EINVAL, "rm_tmem must be -1 (auto), 0 or 1");
         h->opt_rm_tmem = int(value);

@@ -98,6 +98,9 @@ struct bsrng {
     // next sector then finds its 128 B line resident; Grain C2 11.5 vs 10.5
     // Tb/s) or evict-first (0)
     int opt_rm_l2last = 1;
+    // writer-warp kernel: staggered 64 B flush periods per warp-unit (-1 auto:
+    // on when rows are not 16 B aligned, e.g. the paper's 552 B rows)
+    int opt_rm_phase = -1;
     // init: slicing fused into the init kernel (1) or the ballot slice kernels (0)
     int opt_init_fused = 1;
 };

@@ -134,6 +134,9 @@ struct KsArgs {
     int tmem_dbl;
     // ROW_MAJOR 32 B flushes (TMA / 8 B sector stores): L2 evict_last hint
     int l2last;
+    // writer-warp kernel: stagger the units' 64 B flush periods (rowmajor_ws.cuh
+    // ws::phase) so that they do not all flush in the same block
+    int rm_phase;
     uint64_t tma_groups;
     CUtensorMap tmap;  // 3-D view of `out`: [q 32][group][byte], see bsrng.cu
 };
@@ -473,14 +476,24 @@ __device__ __forceinline__ uint64_t l2_evict_last_policy()
     asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
     return p;
 }
+// WS_EXPERIMENT_NO_STG (measurement builds only, no output): the hinted
+// flush stores keep their operands live but issue nothing, which separates
+// the flush's TMEM read-back / address work from its DRAM writes
+#ifdef WS_EXPERIMENT_NO_STG
+#define BSK_NO_STG_RETURN(...) do { asm volatile("" ::__VA_ARGS__); return; } while (0)
+#else
+#define BSK_NO_STG_RETURN(...) do { } while (0)
+#endif
 __device__ __forceinline__ void st128_hint(uint8_t* p, uint32_t a, uint32_t b, uint32_t c, uint32_t d, uint64_t pol)
 {
+    BSK_NO_STG_RETURN("l"(p), "r"(a), "r"(b), "r"(c), "r"(d));
     asm volatile("st.global.L2::cache_hint.v4.u32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(p), "r"(a), "r"(b), "r"(c),
                  "r"(d), "l"(pol)
                  : "memory");
 }
 __device__ __forceinline__ void st64_hint(uint8_t* p, uint32_t a, uint32_t b, uint64_t pol)
 {
+    BSK_NO_STG_RETURN("l"(p), "r"(a), "r"(b));
     asm volatile("st.global.L2::cache_hint.v2.u32 [%0], {%1, %2}, %3;" ::"l"(p), "r"(a), "r"(b), "l"(pol) : "memory");
 }
 // 8 B sector-flush store: evict-first (streaming), or with an L2 evict_last
@@ -703,6 +716,7 @@ __device__ __forceinline__ void rowmajor_store_tmem_wide(uint32_t tm, uint8_t* c
 
 __device__ __forceinline__ void st32_hint(uint8_t* p, uint32_t a, uint64_t pol)
 {
+    BSK_NO_STG_RETURN("l"(p), "r"(a));
     asm volatile("st.global.L2::cache_hint.u32 [%0], %1, %2;" ::"l"(p), "r"(a), "l"(pol) : "memory");
 }
 // Store the run of slots [m0, m1] (0 <= m0, m1 <= 3; empty if m0 > m1) of one

@@ -81,6 +81,9 @@ int launch_keystream(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st)
     a.units = h->units;
     a.scratch = h->sched + 1 + h->units;
     a.l2last = h->opt_rm_l2last;
+    // staggered flush periods in the writer-warp kernel: auto = rows that are
+    // not 16 B aligned (their pieces need 8 B stores whatever the phase)
+    a.rm_phase = h->opt_rm_phase < 0 ? int(a.row_bytes % 16 != 0) : h->opt_rm_phase;
 
     int block = KS_BLOCK, compute_warps = KS_BLOCK / 32;
     size_t smem = RM ? size_t(KS_BLOCK / 32) * bsk::rm_warp_words(U, 8, true) * 4 : 0;

@@ -49,6 +49,16 @@ constexpr uint32_t NSLOT = 16;              // 32-clock blocks per 64 B row piec
 #define WRITER_SLEEP_NS 200
 #endif
 
+// Flush-period phase of a warp-unit (rm_phase): unit u's 64 B row pieces
+// start at blocks B with (B + phase(u)) % NSLOT == 0.  Without it all units
+// flush in the same block: at the paper shape (2^19 instances, one clock-loop
+// warp per SMSP) 512 writers then issue 32 MB of scattered row stores at once
+// every 512 clocks, and the clock-loop warps' per-clock STS queue behind those
+// STGs (a build without the global stores, WS_EXPERIMENT_NO_STG, ran 25%
+// faster; DESIGN.md sec. 5 "ROW_MAJOR output").  Eight even phases: the wide
+// flush needs 8 B aligned pieces; used when rows are not 16 B aligned anyway.
+__device__ __forceinline__ uint32_t phase(int on, uint64_t unit) { return on ? 2u * uint32_t(unit & 7u) : 0u; }
+
 struct Meta {
     uint64_t unit;   // warp-unit of the item (32 groups)
     uint64_t B;      // call-relative index of this 32-clock block
@@ -188,7 +198,7 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
                 const uint32_t pv = warp_volatile(), b = sq % ws::NZ;
                 if (laneid_volatile() == 0) {
                     const uint64_t B = s_b0[pv] + blk;
-                    const uint32_t kk = uint32_t(B % ws::NSLOT);
+                    const uint32_t kk = uint32_t((B + ws::phase(a.rm_phase, s_unit[pv])) % ws::NSLOT);
                     ws::Meta& m = meta[pv][b];
                     m.unit = s_unit[pv];
                     m.B = B;
@@ -259,7 +269,7 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
             if (flags & ws::F_TERM) break;
             const uint64_t unit = vm.unit, B = vm.B;
             const uint32_t k_lo = vm.k_lo;
-            const uint32_t k = uint32_t(B % ws::NSLOT);
+            const uint32_t k = uint32_t((B + ws::phase(a.rm_phase, unit)) % ws::NSLOT);
             const uint32_t tm = *reinterpret_cast<volatile uint32_t*>(&s_tmem) + (pair << 21);
             // WS_EXPERIMENT_NO_WRITER (measurement builds only, wrong output):
             // the writer skips its transposes and flushes, which isolates the

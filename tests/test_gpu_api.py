@@ -89,7 +89,7 @@ def test_option_validation():
     keys, ivs = inputs.make_inputs("grain", 32)
     g = bsrng.Generator("grain", keys, ivs)
     for k, v in (("unroll", 4), ("unroll", 8), ("sched", 2), ("seg_clocks", 33), ("ctas_per_sm", 99), ("rm_ws", 5), ("rm_ws", 3),
-                 ("rm_slots", 4), ("rm_zreg", 0), ("rm_tmem", 2), ("rm_tma", 2), ("rm_dbl", 2), ("init_fused", 2)):
+                 ("rm_slots", 4), ("rm_zreg", 0), ("rm_tmem", 2), ("rm_tma", 2), ("rm_dbl", 2), ("rm_phase", 2), ("rm_phase", -2), ("init_fused", 2)):
         with pytest.raises(bsrng.BsrngError) as e:
             g.set_option(k, v)
         assert e.value.code == bsrng.EINVAL
@@ -162,6 +162,10 @@ def test_mickey_2_40_limit_boundary():
     ("grain", {"rm_ws": 0, "rm_l2last": 0, "rm_tma": 0}, 8192),        # evict-first 8 B sector flush
     ("grain", {"rm_ws": 1}, 4416),                         # writer warp, 552 B rows (STG.64 pieces)
     ("grain", {"rm_ws": 1, "seg_clocks": 512}, 4096 + 1024),
+    ("grain", {"rm_ws": 1, "rm_phase": 0}, 4416),         # 552 B rows, all units flush in the same block
+    ("grain", {"rm_ws": 1, "rm_phase": 1}, 8192),         # staggered flush periods on 16 B-aligned rows
+    ("grain", {"rm_ws": 1, "rm_phase": 1, "seg_clocks": 1056}, 4416 + 96),  # ... and mid-period item starts
+    ("mickey2", {"rm_ws": 1, "rm_phase": 1}, 2048 + 96),
     ("mickey2", {"rm_ws": 1}, 4416),
     # LFSR writer-warp kernel: 128-clock period bodies plus per-clock remainders
     ("lfsr128", {}, 8192),

@@ -21,9 +21,10 @@ from paper_conf_icppw_monfaredhkzrg20_b200 import bsrng, inputs  # noqa: E402
 W = {"rm_ws": 0}
 OPTS = {
     "mickey2": [{}, {"sched": 0}, {**W, "rm_tmem": 0}, W, {**W, "rm_tma": 0}, {**W, "rm_wide": 1},
-                {"seg_clocks": 96}, {**W, "ctas_per_sm": 1}, {**W, "rm_l2last": 0}],
+                {"seg_clocks": 96}, {**W, "ctas_per_sm": 1}, {**W, "rm_l2last": 0}, {"rm_ws": 1, "rm_phase": 1}],
     "grain": [{}, {"sched": 0}, {**W, "rm_tmem": 0}, {"rm_ws": 1}, W, {**W, "rm_tma": 0}, {**W, "rm_wide": 1},
-              {"unroll": 16}, {"seg_clocks": 160}, {"ctas_per_sm": 1}, {**W, "rm_dbl": 0}],
+              {"unroll": 16}, {"seg_clocks": 160}, {"ctas_per_sm": 1}, {**W, "rm_dbl": 0}, {"rm_ws": 1, "rm_phase": 1},
+              {"rm_ws": 1, "rm_phase": 0}],
     "lfsr128": [{}, {"sched": 0}, {"rm_ws": 0}, {"rm_ws": 1}, {"rm_ws": 2}, {"rm_ws": 2, "seg_clocks": 96}, {**W, "rm_wide": 1},
                 {"unroll": 16}, {"seg_clocks": 64}],
     "aes128ctr": [{}, {"rm_ws": 0}, {"ctas_per_sm": 1}, {"seg_clocks": 256}],
