@@ -402,6 +402,35 @@ __device__ __forceinline__ void rowmajor_transpose_smem_tmem(const uint32_t* zs,
     }
 }
 
+// The same from the writer-warp kernels' lane-major z block (rowmajor_ws.cuh
+// ws::ZP): zl = this thread's 32 words (clock t at zl[t], 16 B aligned), read
+// with 8 LDS.128 once for both 16-row halves.
+template <bool MSB_FIRST, int RS>
+__device__ __forceinline__ void rowmajor_transpose_lanes_tmem(const uint32_t* zl, uint32_t tm, uint32_t k)
+{
+    constexpr int X = MSB_FIRST ? 7 : 0;
+    uint32_t w[32];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+        const uint4 v = *reinterpret_cast<const uint4*>(zl + 4 * i);
+        w[4 * i] = v.x;
+        w[4 * i + 1] = v.y;
+        w[4 * i + 2] = v.z;
+        w[4 * i + 3] = v.w;
+    }
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+        uint32_t x[16];
+#pragma unroll
+        for (int q = 0; q < 16; ++q) x[q] = __byte_perm(w[q ^ X], w[(q + 16) ^ X], h == 0 ? 0x5410 : 0x7632);
+        bt_transpose16(x);
+        if (h == 0)
+            tmem_st_rows<0, RS>(tm + k, x, std::make_integer_sequence<int, 16>{});
+        else
+            tmem_st_rows<1, RS>(tm + k, x, std::make_integer_sequence<int, 16>{});
+    }
+}
+
 // Flush slots [k_lo, k_hi] of every real row from TMEM (rowmajor_store's
 // contract).  The loads are warp-collective, so every lane runs all of them;
 // the per-lane row count only predicates the global stores.

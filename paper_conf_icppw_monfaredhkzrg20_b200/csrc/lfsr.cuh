@@ -82,8 +82,8 @@ struct Lfsr128 {
     template <int J, class F>
     __device__ __forceinline__ void period_block(F&& put)
     {
-#pragma unroll
-        for (int u = 0; u < 32; ++u) put(u, s[32 * J + u]);
+        // u as a compile-time constant (the writer-warp kernels group 4 per STS.128)
+        static_for<32>([&](auto u) { put(u, s[32 * J + decltype(u)::value]); });
 #pragma unroll
         for (int t = 32 * J; t < 32 * J + 32; ++t)
             s[t] = lop3<0x96u>(lop3<0x96u>(s[(t + 29) & 127], s[(t + 27) & 127], s[(t + 2) & 127]), s[t], 0u);

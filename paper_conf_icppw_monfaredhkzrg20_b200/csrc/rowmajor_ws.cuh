@@ -32,7 +32,14 @@ namespace ws {
 
 constexpr int NCOMP = 4;                    // compute warps per CTA (one per SMSP)
 constexpr int BLOCK = 2 * NCOMP * 32;       // + one writer warp each
-constexpr int ZBUF = 32 * 32;               // words in one z block: [t][lane]
+// z block layout of the writer-warp kernels: lane L's 32 slice words (clock t
+// at word t) at L * ZP.  The clock-loop warp stores 4 clocks per STS.128 and
+// the writer loads its lane's 32 words with 8 LDS.128, both bank-conflict free
+// at ZP = 36 (an 8-lane store phase covers all 32 banks).  One STS.32 per
+// clock ([t][lane] layout) put 4x the shared-memory instructions into the MIO
+// queue the writers' flush STGs also use.
+constexpr int ZP = 36;
+constexpr int ZBUF = 32 * ZP;               // words in one z block: [lane][ZP]
 #ifndef WS_NZ
 #define WS_NZ 8
 #endif
@@ -43,7 +50,7 @@ constexpr int NZ = WS_NZ;                   // z blocks in flight per pair (abso
 constexpr int G = WS_G;                     // z blocks per empty-barrier wait of the clock-loop warp
 static_assert(G >= 1 && G <= NZ, "a wait group must fit in the ring");
 constexpr int PAIR_WORDS = NZ * ZBUF;
-constexpr size_t SMEM_BYTES = size_t(NCOMP) * PAIR_WORDS * 4;  // 4 KB per z block: 128 KB
+constexpr size_t SMEM_BYTES = size_t(NCOMP) * PAIR_WORDS * 4;  // 4.5 KB per z block: 144 KB
 constexpr uint32_t NSLOT = 16;              // 32-clock blocks per 64 B row piece
 #ifndef WRITER_SLEEP_NS
 #define WRITER_SLEEP_NS 200
@@ -66,6 +73,15 @@ struct Meta {
     uint32_t flags;  // F_FLUSH | F_TERM
 };
 enum : uint32_t { F_FLUSH = 1u, F_TERM = 2u };
+
+// Store z words of 4 consecutive clocks (u = 4m .. 4m+3 of a block) with one
+// STS.128: zz collects them, the 4th clock's call stores.
+template <int UU>
+__device__ __forceinline__ void put_z4(uint32_t* zl, uint32_t (&zz)[4], uint32_t v)
+{
+    zz[UU & 3] = v;
+    if constexpr ((UU & 3) == 3) *reinterpret_cast<uint4*>(zl + (UU & ~3)) = make_uint4(zz[0], zz[1], zz[2], zz[3]);
+}
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p)
 {
@@ -116,10 +132,10 @@ __device__ __forceinline__ void mbar_wait_sleepy(uint64_t* bar, uint32_t parity)
 template <class C, int U>
 __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __grid_constant__ KsArgs a)
 {
-    static_assert(32 % U == 0, "U must divide 32");
+    static_assert(32 % U == 0 && U % 4 == 0, "U must divide 32 (and hold whole STS.128 groups)");
     constexpr int KB = ks_block<C, U>();
     static_assert(U % KB == 0, "the loop body must hold whole schedule blocks");
-    extern __shared__ uint32_t pair_smem[];  // [NCOMP][NZ z blocks]
+    extern __shared__ __align__(16) uint32_t pair_smem[];  // [NCOMP][NZ z blocks]
     __shared__ uint64_t bar_full[ws::NCOMP][ws::NZ], bar_empty[ws::NCOMP][ws::NZ];
     __shared__ ws::Meta meta[ws::NCOMP][ws::NZ];
     __shared__ uint32_t s_item[ws::NCOMP];
@@ -178,7 +194,7 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
             // ring slot of z block sq (its empty barrier already waited for)
             auto slot_ptr = [&](uint32_t sq) {
                 const uint32_t pv = warp_volatile(), b = sq % ws::NZ;
-                return pair_smem + pv * ws::PAIR_WORDS + b * ws::ZBUF + laneid_volatile();
+                return pair_smem + pv * ws::PAIR_WORDS + b * ws::ZBUF + laneid_volatile() * ws::ZP;
             };
             // The writer consumes z blocks in order, so slot sq's empty barrier
             // having completed its phase implies the same for every earlier
@@ -217,7 +233,8 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
                     static_for<PB>([&](auto jj) {
                         constexpr int J = decltype(jj)::value;
                         uint32_t* zb = acquire(seq + J);
-                        c.template period_block<J>([&](int u, uint32_t v) { zb[u * 32] = v; });
+                        uint32_t zz[4];
+                        c.template period_block<J>([&](auto u, uint32_t v) { ws::put_z4<decltype(u)::value>(zb, zz, v); });
                         publish(seq + J, blk + J);
                     });
                 }
@@ -231,9 +248,10 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
                     uint32_t* zb = slot_ptr(seq);
 #pragma unroll 1
                     for (uint32_t k = 0; k < 32; k += U) {
+                        uint32_t zz[4];
                         static_for<U>([&](auto u) {
                             constexpr int J = decltype(u)::value % KB;
-                            zb[(k + decltype(u)::value) * 32] = ks_z<J, KB>(c);
+                            ws::put_z4<decltype(u)::value>(zb + k, zz, ks_z<J, KB>(c));
                             ks_clock<J, KB>(c);
                         });
                     }
@@ -275,7 +293,7 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
             // the writer skips its transposes and flushes, which isolates the
             // lone clock-loop warp's own rate
 #ifndef WS_EXPERIMENT_NO_WRITER
-            rowmajor_transpose_smem_tmem<C::MSB_FIRST, 16>(zbase + b * ws::ZBUF + lane, tm, wide_col(k));
+            rowmajor_transpose_lanes_tmem<C::MSB_FIRST, 16>(zbase + b * ws::ZBUF + lane * ws::ZP, tm, wide_col(k));
 #endif
             ws::mbar_arrive(&bar_empty[pair][b]);
 #if defined(WS_EXPERIMENT_NO_WRITER) || defined(WS_EXPERIMENT_NO_FLUSH)

@@ -41,14 +41,14 @@ namespace ws2 {
 constexpr int NSTREAM = 2;                      // clock-loop warps per CTA (warps 4, 5)
 constexpr int NWRITER = 4;                      // writer warps 0..3 (lane quarter = warp index)
 constexpr int BLOCK = (NWRITER + NSTREAM) * 32;
-constexpr int ZBUF = 32 * 32;                   // words in one z block: [t][lane]
+constexpr int ZBUF = ws::ZBUF;                  // words in one z block: [lane][ws::ZP]
 #ifndef WS2_NZ
 #define WS2_NZ 24
 #endif
 // ring slots per stream (multiple of 8): block seq -> slot seq % NZ, owner (seq >> 3) & 1
 constexpr int NZ = WS2_NZ;
 static_assert(NZ % 8 == 0 && NZ >= 16, "whole 8-block owner groups, at least one per writer");
-constexpr size_t SMEM_BYTES = size_t(NSTREAM) * NZ * ZBUF * 4;  // 192 KB at NZ = 24
+constexpr size_t SMEM_BYTES = size_t(NSTREAM) * NZ * ZBUF * 4;  // 216 KB at NZ = 24
 constexpr uint32_t PERIOD = 32;                 // 32-clock blocks per 128 B row piece
 
 struct Meta {
@@ -175,7 +175,7 @@ __global__ void __launch_bounds__(ws2::BLOCK, 1) keystream_rm_ws2_kernel(const _
         // (kept out of the register-saturated clock loop, rowmajor_ws.cuh)
         auto sidv = [&]() { return warp_volatile() - uint32_t(ws2::NWRITER); };
         auto slot_ptr = [&](uint32_t sq) {
-            return ring_smem + (sidv() * ws2::NZ + sq % ws2::NZ) * ws2::ZBUF + laneid_volatile();
+            return ring_smem + (sidv() * ws2::NZ + sq % ws2::NZ) * ws2::ZBUF + laneid_volatile() * ws::ZP;
         };
         // (backs off while waiting: the writer it waits for may share its SMSP)
         auto wait_empty = [&](uint32_t sq) {
@@ -253,7 +253,8 @@ __global__ void __launch_bounds__(ws2::BLOCK, 1) keystream_rm_ws2_kernel(const _
                         constexpr int J = decltype(jj)::value;
                         if (!grouped) wait_empty(seq + J);
                         uint32_t* zb = slot_ptr(seq + J);
-                        c.template period_block<J>([&](int u, uint32_t v) { zb[u * 32] = v; });
+                        uint32_t zz[4];
+                        c.template period_block<J>([&](auto u, uint32_t v) { ws::put_z4<decltype(u)::value>(zb, zz, v); });
                         publish(seq + J, blk + J);
                     });
                 }
@@ -264,9 +265,10 @@ __global__ void __launch_bounds__(ws2::BLOCK, 1) keystream_rm_ws2_kernel(const _
                 uint32_t* zb = slot_ptr(seq);
 #pragma unroll 1
                 for (uint32_t k = 0; k < 32; k += U) {
+                    uint32_t zz[4];
                     static_for<U>([&](auto u) {
                         constexpr int J = decltype(u)::value % KB;
-                        zb[(k + decltype(u)::value) * 32] = ks_z<J, KB>(c);
+                        ws::put_z4<decltype(u)::value>(zb + k, zz, ks_z<J, KB>(c));
                         ks_clock<J, KB>(c);
                     });
                 }
@@ -318,7 +320,7 @@ __global__ void __launch_bounds__(ws2::BLOCK, 1) keystream_rm_ws2_kernel(const _
             const uint32_t k = uint32_t(B % ws2::PERIOD);
             const uint32_t kl = 8 * (k >> 4) + (k & 7u);  // local slot in this writer's quarter
             const uint32_t tm = *reinterpret_cast<volatile uint32_t*>(&s_tmem) + (warp << 21);
-            rowmajor_transpose_smem_tmem<C::MSB_FIRST, 16>(zbase + b * ws2::ZBUF + lane, tm, wide_col(kl));
+            rowmajor_transpose_lanes_tmem<C::MSB_FIRST, 16>(zbase + b * ws2::ZBUF + lane * ws::ZP, tm, wide_col(kl));
             ws::mbar_arrive(&bar_empty[sid][b]);
             if (flags & ws2::F_FLUSH) {
                 const uint64_t first = (unit * 32u + lane) * 32u;
