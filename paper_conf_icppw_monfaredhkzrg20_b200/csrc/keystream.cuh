@@ -431,6 +431,53 @@ __device__ __forceinline__ void rowmajor_transpose_lanes_tmem(const uint32_t* zl
     }
 }
 
+// Two consecutive blocks of the same rows (slots k, k + 1 at adjacent
+// columns, k even under wide_col): both transposes interleaved (twice the
+// independent work for a lone writer warp) and each row's two words written
+// by one tcgen05.st.32x32b.x2 -- 32 instead of 64 STTM per pair (ptxas also
+// emitted one R2UR per STTM).
+template <int OFF>
+__device__ __forceinline__ void tmem_st2(uint32_t taddr, uint32_t v0, uint32_t v1)
+{
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x2.b32 [%0+%3], {%1, %2};" ::"r"(taddr), "r"(v0), "r"(v1), "n"(OFF)
+                 : "memory");
+}
+template <int H, int RS, int... Q>
+__device__ __forceinline__ void tmem_st_rows2(uint32_t base, const uint32_t (&x0)[16], const uint32_t (&x1)[16],
+                                              std::integer_sequence<int, Q...>)
+{
+    (tmem_st2<(16 * H + Q) * RS>(base, x0[Q], x1[Q]), ...);
+}
+template <bool MSB_FIRST, int RS>
+__device__ __forceinline__ void rowmajor_transpose_lanes_tmem2(const uint32_t* zl0, const uint32_t* zl1, uint32_t tm,
+                                                               uint32_t k)
+{
+    constexpr int X = MSB_FIRST ? 7 : 0;
+    uint32_t w0[32], w1[32];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+        const uint4 v = *reinterpret_cast<const uint4*>(zl0 + 4 * i);
+        const uint4 u = *reinterpret_cast<const uint4*>(zl1 + 4 * i);
+        w0[4 * i] = v.x, w0[4 * i + 1] = v.y, w0[4 * i + 2] = v.z, w0[4 * i + 3] = v.w;
+        w1[4 * i] = u.x, w1[4 * i + 1] = u.y, w1[4 * i + 2] = u.z, w1[4 * i + 3] = u.w;
+    }
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+        uint32_t x0[16], x1[16];
+#pragma unroll
+        for (int q = 0; q < 16; ++q) {
+            x0[q] = __byte_perm(w0[q ^ X], w0[(q + 16) ^ X], h == 0 ? 0x5410 : 0x7632);
+            x1[q] = __byte_perm(w1[q ^ X], w1[(q + 16) ^ X], h == 0 ? 0x5410 : 0x7632);
+        }
+        bt_transpose16(x0);
+        bt_transpose16(x1);
+        if (h == 0)
+            tmem_st_rows2<0, RS>(tm + k, x0, x1, std::make_integer_sequence<int, 16>{});
+        else
+            tmem_st_rows2<1, RS>(tm + k, x0, x1, std::make_integer_sequence<int, 16>{});
+    }
+}
+
 // Flush slots [k_lo, k_hi] of every real row from TMEM (rowmajor_store's
 // contract).  The loads are warp-collective, so every lane runs all of them;
 // the per-lane row count only predicates the global stores.

@@ -43,12 +43,12 @@ constexpr int NWRITER = 4;                      // writer warps 0..3 (lane quart
 constexpr int BLOCK = (NWRITER + NSTREAM) * 32;
 constexpr int ZBUF = ws::ZBUF;                  // words in one z block: [lane][ws::ZP]
 #ifndef WS2_NZ
-#define WS2_NZ 24
+#define WS2_NZ 16
 #endif
 // ring slots per stream (multiple of 8): block seq -> slot seq % NZ, owner (seq >> 3) & 1
 constexpr int NZ = WS2_NZ;
 static_assert(NZ % 8 == 0 && NZ >= 16, "whole 8-block owner groups, at least one per writer");
-constexpr size_t SMEM_BYTES = size_t(NSTREAM) * NZ * ZBUF * 4;  // 216 KB at NZ = 24
+constexpr size_t SMEM_BYTES = size_t(NSTREAM) * NZ * ZBUF * 4;  // 144 KB at NZ = 16
 constexpr uint32_t PERIOD = 32;                 // 32-clock blocks per 128 B row piece
 
 struct Meta {
@@ -57,8 +57,13 @@ struct Meta {
     uint32_t k_lo;   // first period slot of the item in this period
     uint32_t flags;  // F_FLUSH | F_TERM | F_SKIP
 };
-enum : uint32_t { F_FLUSH = 1u, F_TERM = 2u, F_SKIP = 4u };
+// F_PAIR: an even block whose successor is the same item's next block (the
+// writer transposes the two together)
+enum : uint32_t { F_FLUSH = 1u, F_TERM = 2u, F_SKIP = 4u, F_PAIR = 8u };
 
+#ifndef WS2_BACKOFF_NS
+#define WS2_BACKOFF_NS 64
+#endif
 // try_wait with a short back-off once the first probe fails
 __device__ __forceinline__ void mbar_wait_backoff(uint64_t* bar, uint32_t parity)
 {
@@ -72,7 +77,7 @@ __device__ __forceinline__ void mbar_wait_backoff(uint64_t* bar, uint32_t parity
             : "r"(ws::smem_u32(bar)), "r"(parity)
             : "memory");
         if (ok) break;
-        __nanosleep(64);
+        __nanosleep(WS2_BACKOFF_NS);
     }
 }
 
@@ -237,7 +242,7 @@ __global__ void __launch_bounds__(ws2::BLOCK, 1) keystream_rm_ws2_kernel(const _
                     m.unit = s_unit[sv];
                     m.B = B;
                     m.k_lo = k - (blk < k ? blk : k);
-                    m.flags = fl ? ws2::F_FLUSH : 0u;
+                    m.flags = (fl ? ws2::F_FLUSH : 0u) | ((B & 1u) == 0 && blk + 1 < nblk ? ws2::F_PAIR : 0u);
                 }
                 ws::mbar_arrive(&bar_full[sv][b]);
             };
@@ -319,6 +324,39 @@ __global__ void __launch_bounds__(ws2::BLOCK, 1) keystream_rm_ws2_kernel(const _
             const volatile ws2::Meta& vm = meta[sid][b];
             const uint32_t flags = vm.flags;
             if (flags & ws2::F_TERM) break;
+            // Both blocks of a pair consecutive blocks of one item (F_PAIR): they
+            // sit at consecutive local slots (seq = B (mod 16), B even, kl even)
+            // and the first one does not end the writer's period (only an item's
+            // last block would).  One paired transpose.
+            if ((i & 1u) == 0 && (flags & ws2::F_PAIR)) {
+                const uint32_t b1 = (sq + 1) % ws2::NZ;
+                const volatile ws2::Meta& vm1 = meta[sid][b1];
+                const uint32_t flags1 = vm1.flags;
+                {
+                    const uint64_t unit = vm1.unit, B = vm1.B;
+                    const uint32_t k_lo = vm1.k_lo;
+                    const uint32_t k = uint32_t(B % ws2::PERIOD);
+                    const uint32_t kl = 8 * (k >> 4) + (k & 7u) - 1;  // the pair's first (even) local slot
+                    const uint32_t tm = *reinterpret_cast<volatile uint32_t*>(&s_tmem) + (warp << 21);
+                    rowmajor_transpose_lanes_tmem2<C::MSB_FIRST, 16>(zbase + b * ws2::ZBUF + lane * ws::ZP,
+                                                                     zbase + b1 * ws2::ZBUF + lane * ws::ZP, tm,
+                                                                     wide_col(kl));
+                    ws::mbar_arrive(&bar_empty[sid][b]);
+                    ws::mbar_arrive(&bar_empty[sid][b1]);
+                    ++i;  // the pair's second block is done as well
+                    if (flags1 & ws2::F_FLUSH) {
+                        const uint64_t first = (unit * 32u + lane) * 32u;
+                        const uint32_t nvalid = first >= a.n ? 0u : uint32_t(a.n - first < 32 ? a.n - first : 32);
+                        s_row0[warp][lane] = static_cast<uint8_t*>(a.out) + (nvalid ? first : 0) * a.row_bytes;
+                        s_nvalid[warp][lane] = nvalid;
+                        __syncwarp();
+                        const uint64_t col = (B - (k - k_lo)) * 4;
+                        ws2::store_split(tm, s_row0[warp], s_nvalid[warp], a.row_bytes, wr, k_lo, k, col);
+                        __syncwarp();
+                    }
+                    continue;
+                }
+            }
             if (flags & ws2::F_SKIP) {
                 ws::mbar_arrive(&bar_empty[sid][b]);
                 continue;

@@ -1,9 +1,8 @@
 #!/bin/bash
-# lane-major z blocks (STS.128 / LDS.128) in the writer-warp kernels: parity, then A/B vs the
-# previous build (tools/experiments/ab/old.so) on the writer-warp workloads
+# ws2 writer: paired-block transposes (STTM.x2).  Parity, then A/B vs HEAD with NZ = 16 (nz16.so).
 set -u
-D=gpurun_out/g7; mkdir -p $D
-timeout 900 python -m pytest tests/test_gpu_api.py tests/test_gpu_random.py tests/test_gpu_rowmajor_items.py tests/test_gpu_lfsr.py -m gpu -q -x -p no:cacheprovider > $D/pytest.txt 2>&1
+D=gpurun_out/g14; mkdir -p $D
+timeout 900 python -m pytest tests/test_gpu_api.py tests/test_gpu_random.py tests/test_gpu_rowmajor_items.py tests/test_gpu_lfsr.py -m gpu -q -p no:cacheprovider > $D/pytest.txt 2>&1
 echo "pytest exit $?" >> $D/pytest.txt
 run() {  # name lib args...
   local name=$1 lib=$2; shift 2
@@ -11,11 +10,6 @@ run() {  # name lib args...
   python -c "import json; d=json.load(open('$D/$name.json')); print('$name', round(d['value'],3), d['modes']['materialise']['kernel_ms_per_step'])" >> $D/summary.txt 2>&1
 }
 for rep in 1 2; do
-  for v in new old; do
-    lib=""; [ $v = old ] && lib=tools/experiments/ab/old.so
-    run c4_grain_$v "$lib" --cipher grain --workload c4 --steps 1000 --warmup 20
-    run c4_mickey_$v "$lib" --cipher mickey2 --workload c4 --steps 300 --warmup 10
-    run lfsr_ws2_$v "$lib" --cipher lfsr128 --steps 20 --warmup 3
-    run lfsr_ws1_$v "$lib" --cipher lfsr128 --steps 20 --warmup 3 --opt rm_ws=1
-  done
+  run lfsr_new "" --cipher lfsr128 --steps 20 --warmup 3
+  run lfsr_nz16 tools/experiments/ab/nz16.so --cipher lfsr128 --steps 20 --warmup 3
 done
