@@ -25,7 +25,8 @@ cases = [
     ("grain", 32 * 40 + 9, 1024 + 512, {**W, "rm_wide": 1}), ("grain", 32 * 40 + 9, 1024, {**W, "rm_tma": 0}),
     ("aes128ctr", 32 * 9 + 5, 4480, {}), ("aes128ctr", 32 * 9 + 5, 4480, {"rm_ws": 0}),
     ("lfsr128", 32 * 37 + 13, 1024, {}), ("lfsr128", 32 * 37 + 13, 2048 + 96, {}),    # period bodies + remainder
-    ("lfsr128", 32 * 37 + 13, 1024, {"rm_ws": 0}),
+    ("lfsr128", 32 * 37 + 13, 1024, {"rm_ws": 0}), ("lfsr128", 32 * 37 + 13, 1024, {"rm_ws": 1}),
+    ("lfsr128", 32 * 37 + 13, 3200, {"seg_clocks": 160}),   # two-writer kernel: odd item starts, unpaired blocks
 ]
 # synccheck stops the process at the plain TMEM kernel ("Barrier error
 # detected. Missing init" at shared address 0x0, PC outside the kernel; see
