@@ -127,3 +127,30 @@ def test_rowmajor_lanes_plus_remainder(bits):
     got2 = g.generate_host(bits, "row_major")
     assert np.array_equal(got1, want[:, :bits // 8])
     assert np.array_equal(got2, want[:, bits // 8:])
+
+
+@pytest.mark.parametrize("device_inputs", [False, True])
+@pytest.mark.parametrize("bits", [4096 + 384, 4096 + 31 * 128, 8192 + 128])
+def test_rowmajor_remainder_pairs_carries(bits, device_inputs):
+    """Block-lane ROW_MAJOR calls with a < 32-block remainder per row (the
+    instance-sliced kernel writes the rows' last blocks): counters whose block
+    index carries through the low 32 and 64 bits and wraps at 2^128 inside the
+    remainder, a second call (block indices offset by the first call), ragged
+    n, host and device-resident counters."""
+    n = 32 * 7 + 19
+    _, ctrs = inputs.make_inputs("aes128ctr", n, seed=77)
+    ctrs = ctrs.copy()
+    ctrs[3] = np.frombuffer(bytes([0xFF] * 16), np.uint8)                        # wraps at the first block
+    ctrs[4, 12:] = 0xFF                                                          # low word carries
+    ctrs[5, 8:] = 0xFF
+    ctrs[5, 15] = 0xDF                                                           # carry out of 64 bits mid-row
+    ctrs[33] = np.frombuffer(bytes([0xFF] * 15 + [0xD8]), np.uint8)              # 128-bit wrap inside the remainder
+    key = inputs.aes_key(5)
+    if device_inputs:
+        g = bsrng.Generator("aes128ctr", torch.from_numpy(key).cuda(), torch.from_numpy(ctrs).cuda())
+    else:
+        g = bsrng.Generator("aes128ctr", key, ctrs)
+    want = oracle.aes128_ctr_keystream_batch(bytes(key), ctrs, 2 * bits)
+    for call in range(2):
+        got = g.generate_host(bits, "row_major")
+        assert np.array_equal(got, want[:, call * bits // 8:(call + 1) * bits // 8]), call
