@@ -66,13 +66,21 @@ constexpr uint32_t NSLOT = 16;              // 32-clock blocks per 64 B row piec
 // flush needs 8 B aligned pieces; used when rows are not 16 B aligned anyway.
 __device__ __forceinline__ uint32_t phase(int on, uint64_t unit) { return on ? 2u * uint32_t(unit & 7u) : 0u; }
 
-struct Meta {
-    uint64_t unit;   // warp-unit of the item (32 groups)
-    uint64_t B;      // call-relative index of this 32-clock block
-    uint32_t k_lo;   // first staged slot to write on flush
-    uint32_t flags;  // F_FLUSH | F_TERM
+// One record per work item (not per block): the clock-loop warp writes it at
+// the item's start, before it arrives on the item's first z block; the writer
+// derives every block's period slot and flush flag from it.  Per-block meta
+// written by lane 0 (a divergent section with two dependent shared loads)
+// cost the lone clock-loop warp 6.4% of its time at the paper shape (Grain,
+// measured with a build that skipped those writes).  nblk == 0 terminates.
+struct Item {
+    uint64_t unit;  // warp-unit (32 groups)
+    uint64_t b0;    // call-relative index of the item's first 32-clock block
+    uint32_t nblk;  // blocks in the item
+    uint32_t pad;
 };
-enum : uint32_t { F_FLUSH = 1u, F_TERM = 2u };
+constexpr int NITEM = 16;  // records in flight per pair (> NZ + 1: the writer lags at most NZ blocks)
+static_assert(NITEM > NZ + 1, "item ring");
+enum : uint32_t { F_FLUSH = 1u };
 
 // Store z words of 4 consecutive clocks (u = 4m .. 4m+3 of a block) with one
 // STS.128: zz collects them, the 4th clock's call stores.
@@ -137,14 +145,15 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
     static_assert(U % KB == 0, "the loop body must hold whole schedule blocks");
     extern __shared__ __align__(16) uint32_t pair_smem[];  // [NCOMP][NZ z blocks]
     __shared__ uint64_t bar_full[ws::NCOMP][ws::NZ], bar_empty[ws::NCOMP][ws::NZ];
-    __shared__ ws::Meta meta[ws::NCOMP][ws::NZ];
+    __shared__ ws::Item items[ws::NCOMP][ws::NITEM];
     __shared__ uint32_t s_item[ws::NCOMP];
-    __shared__ uint64_t s_unit[ws::NCOMP], s_b0[ws::NCOMP];  // per-item context of each compute warp
+    __shared__ uint32_t s_nitem[ws::NCOMP];  // items started by each compute warp
     __shared__ uint8_t* s_row0[ws::NCOMP][32];                // writer: row bases of the unit's groups
     __shared__ uint32_t s_nvalid[ws::NCOMP][32];
     __shared__ uint32_t s_tmem;
 
     if (threadIdx.x == 0) {
+        for (int c = 0; c < ws::NCOMP; ++c) s_nitem[c] = 0;
         for (int c = 0; c < ws::NCOMP; ++c)
             for (int b = 0; b < ws::NZ; ++b) {
                 ws::mbar_init(&bar_full[c][b], 32);
@@ -182,8 +191,12 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
             const uint32_t nblk = uint32_t((left < a.seg_clocks ? left : a.seg_clocks) >> 5);
 
             if (lane == 0) {
-                s_unit[pair] = w;
-                s_b0[pair] = clk_begin >> 5;
+                const uint32_t ni = s_nitem[pair];
+                ws::Item& it = items[pair][ni % ws::NITEM];
+                it.unit = w;
+                it.b0 = clk_begin >> 5;
+                it.nblk = nblk;
+                s_nitem[pair] = ni + 1;
             }
             C c;
             c.load(a.state, a.Gp, g);
@@ -210,17 +223,9 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
                 wait_empty(sq);
                 return slot_ptr(sq);
             };
-            auto publish = [&](uint32_t sq, uint32_t blk) {
+            // z block sq complete (the writer derives its slot from the item record)
+            auto publish = [&](uint32_t sq, uint32_t) {
                 const uint32_t pv = warp_volatile(), b = sq % ws::NZ;
-                if (laneid_volatile() == 0) {
-                    const uint64_t B = s_b0[pv] + blk;
-                    const uint32_t kk = uint32_t((B + ws::phase(a.rm_phase, s_unit[pv])) % ws::NSLOT);
-                    ws::Meta& m = meta[pv][b];
-                    m.unit = s_unit[pv];
-                    m.B = B;
-                    m.k_lo = kk - (blk < kk ? blk : kk);
-                    m.flags = (kk == ws::NSLOT - 1 || blk + 1 == nblk) ? ws::F_FLUSH : 0u;
-                }
                 ws::mbar_arrive(&bar_full[pv][b]);
             };
             uint32_t blk = 0;
@@ -274,20 +279,30 @@ __global__ void __launch_bounds__(ws::BLOCK, 1) keystream_rm_ws_kernel(const __g
         }
         const uint32_t b = seq % ws::NZ;
         if (seq >= ws::NZ) ws::mbar_wait(&bar_empty[pair][b], ((seq / ws::NZ) - 1) & 1u);
-        if (laneid_volatile() == 0) meta[pair][b].flags = ws::F_TERM;
+        if (laneid_volatile() == 0) items[pair][s_nitem[pair] % ws::NITEM].nblk = 0;  // terminate record
         ws::mbar_arrive(&bar_full[pair][b]);
     } else {
         // ------------------------------------------------------------- writer
         const uint32_t lane = threadIdx.x & 31u;
+        uint64_t unit = 0, b0 = 0;
+        uint32_t nblk = 0, seq0 = 0, nrec = 0;
         for (uint32_t seq = 0;; ++seq) {
             const uint32_t b = seq % ws::NZ;
             ws::mbar_wait_sleepy(&bar_full[pair][b], (seq / ws::NZ) & 1u);
-            const volatile ws::Meta& vm = meta[pair][b];
-            const uint32_t flags = vm.flags;
-            if (flags & ws::F_TERM) break;
-            const uint64_t unit = vm.unit, B = vm.B;
-            const uint32_t k_lo = vm.k_lo;
+            if (seq == seq0 + nblk) {  // the next item's first block (or the terminate marker)
+                const volatile ws::Item& it = items[pair][nrec % ws::NITEM];
+                ++nrec;
+                nblk = it.nblk;
+                if (nblk == 0) break;
+                unit = it.unit;
+                b0 = it.b0;
+                seq0 = seq;
+            }
+            const uint32_t blk = seq - seq0;
+            const uint64_t B = b0 + blk;
             const uint32_t k = uint32_t((B + ws::phase(a.rm_phase, unit)) % ws::NSLOT);
+            const uint32_t k_lo = k - (blk < k ? blk : k);
+            const uint32_t flags = (k == ws::NSLOT - 1 || blk + 1 == nblk) ? ws::F_FLUSH : 0u;
             const uint32_t tm = *reinterpret_cast<volatile uint32_t*>(&s_tmem) + (pair << 21);
             // WS_EXPERIMENT_NO_WRITER (measurement builds only, wrong output):
             // the writer skips its transposes and flushes, which isolates the
