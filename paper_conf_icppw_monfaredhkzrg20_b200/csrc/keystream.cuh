@@ -341,6 +341,12 @@ __device__ __forceinline__ void tmem_st1(uint32_t taddr, uint32_t v)
 {
     asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0+%2], {%1};" ::"r"(taddr), "r"(v), "n"(OFF) : "memory");
 }
+// A TMEM address as a warp-uniform value: ptxas then keeps it in one uniform
+// register and folds the column offsets into the STTMs (STTM tmem[UR+imm]);
+// from a per-thread register it emitted one R2UR per STTM (32 per 32-clock
+// block).
+__device__ __forceinline__ uint32_t tmem_uniform(uint32_t taddr) { return __shfl_sync(0xFFFFFFFFu, taddr, 0); }
+
 template <int H, int RS, int... Q>
 __device__ __forceinline__ void tmem_st_rows(uint32_t base, const uint32_t (&x)[16], std::integer_sequence<int, Q...>)
 {
@@ -378,9 +384,9 @@ __device__ __forceinline__ void rowmajor_transpose_tmem(const uint32_t (&z)[32],
         for (int q = 0; q < 16; ++q) x[q] = __byte_perm(z[q ^ X], z[(q + 16) ^ X], h == 0 ? 0x5410 : 0x7632);
         bt_transpose16(x);
         if (h == 0)
-            tmem_st_rows<0, RS>(tm + k, x, std::make_integer_sequence<int, 16>{});
+            tmem_st_rows<0, RS>(tmem_uniform(tm + k), x, std::make_integer_sequence<int, 16>{});
         else
-            tmem_st_rows<1, RS>(tm + k, x, std::make_integer_sequence<int, 16>{});
+            tmem_st_rows<1, RS>(tmem_uniform(tm + k), x, std::make_integer_sequence<int, 16>{});
     }
 }
 // The same from 32 z words staged in shared memory ([t][lane], zs = lane's column).
@@ -396,9 +402,9 @@ __device__ __forceinline__ void rowmajor_transpose_smem_tmem(const uint32_t* zs,
             x[q] = __byte_perm(zs[(q ^ X) * 32], zs[((q + 16) ^ X) * 32], h == 0 ? 0x5410 : 0x7632);
         bt_transpose16(x);
         if (h == 0)
-            tmem_st_rows<0, RS>(tm + k, x, std::make_integer_sequence<int, 16>{});
+            tmem_st_rows<0, RS>(tmem_uniform(tm + k), x, std::make_integer_sequence<int, 16>{});
         else
-            tmem_st_rows<1, RS>(tm + k, x, std::make_integer_sequence<int, 16>{});
+            tmem_st_rows<1, RS>(tmem_uniform(tm + k), x, std::make_integer_sequence<int, 16>{});
     }
 }
 
@@ -409,6 +415,7 @@ template <bool MSB_FIRST, int RS>
 __device__ __forceinline__ void rowmajor_transpose_lanes_tmem(const uint32_t* zl, uint32_t tm, uint32_t k)
 {
     constexpr int X = MSB_FIRST ? 7 : 0;
+    const uint32_t tmb = tmem_uniform(tm + k);
     uint32_t w[32];
 #pragma unroll
     for (int i = 0; i < 8; ++i) {
@@ -425,9 +432,9 @@ __device__ __forceinline__ void rowmajor_transpose_lanes_tmem(const uint32_t* zl
         for (int q = 0; q < 16; ++q) x[q] = __byte_perm(w[q ^ X], w[(q + 16) ^ X], h == 0 ? 0x5410 : 0x7632);
         bt_transpose16(x);
         if (h == 0)
-            tmem_st_rows<0, RS>(tm + k, x, std::make_integer_sequence<int, 16>{});
+            tmem_st_rows<0, RS>(tmb, x, std::make_integer_sequence<int, 16>{});
         else
-            tmem_st_rows<1, RS>(tm + k, x, std::make_integer_sequence<int, 16>{});
+            tmem_st_rows<1, RS>(tmb, x, std::make_integer_sequence<int, 16>{});
     }
 }
 
@@ -472,9 +479,9 @@ __device__ __forceinline__ void rowmajor_transpose_lanes_tmem2(const uint32_t* z
         bt_transpose16(x0);
         bt_transpose16(x1);
         if (h == 0)
-            tmem_st_rows2<0, RS>(tm + k, x0, x1, std::make_integer_sequence<int, 16>{});
+            tmem_st_rows2<0, RS>(tmem_uniform(tm + k), x0, x1, std::make_integer_sequence<int, 16>{});
         else
-            tmem_st_rows2<1, RS>(tm + k, x0, x1, std::make_integer_sequence<int, 16>{});
+            tmem_st_rows2<1, RS>(tmem_uniform(tm + k), x0, x1, std::make_integer_sequence<int, 16>{});
     }
 }
 

@@ -1,8 +1,8 @@
 #!/bin/bash
-# writer transposes: stage-16 split on the FMA pipe (WS_FMA16).  Parity with that build, A/B.
+# TMEM addresses as warp-uniform values (one UR per transpose, no R2UR per STTM).  Parity, A/B vs HEAD.
 set -u
-D=gpurun_out/g25; mkdir -p $D
-BSRNG_LIB=tools/experiments/ab/fma16.so timeout 900 python -m pytest tests/test_gpu_api.py tests/test_gpu_random.py tests/test_gpu_rowmajor_items.py tests/test_gpu_bounds.py -m gpu -q -p no:cacheprovider > $D/pytest.txt 2>&1
+D=gpurun_out/g26; mkdir -p $D
+timeout 900 python -m pytest tests/test_gpu_api.py tests/test_gpu_random.py tests/test_gpu_rowmajor_items.py tests/test_gpu_bounds.py -m gpu -q -p no:cacheprovider > $D/pytest.txt 2>&1
 echo "pytest exit $?" >> $D/pytest.txt
 run() {  # name lib args...
   local name=$1 lib=$2; shift 2
@@ -10,9 +10,12 @@ run() {  # name lib args...
   python -c "import json; d=json.load(open('$D/$name.json')); print('$name', round(d['value'],3), [m['kernel_ms_per_step'] for m in d['modes'].values() if m])" >> $D/summary.txt 2>&1
 }
 for rep in 1 2; do
-  for v in fma16 old; do
-    run c4_grain_$v tools/experiments/ab/$v.so --mode materialise --cipher grain --workload c4 --steps 1000 --warmup 20
-    run c4_mickey_$v tools/experiments/ab/$v.so --mode materialise --cipher mickey2 --workload c4 --steps 300 --warmup 10
-    run lfsr_$v tools/experiments/ab/$v.so --mode materialise --cipher lfsr128 --steps 20 --warmup 3
+  for v in new old; do
+    lib=""; [ $v = old ] && lib=tools/experiments/ab/old.so
+    run c4_grain_$v "$lib" --mode materialise --cipher grain --workload c4 --steps 1000 --warmup 20
+    run c4_mickey_$v "$lib" --mode materialise --cipher mickey2 --workload c4 --steps 300 --warmup 10
+    run lfsr_$v "$lib" --mode materialise --cipher lfsr128 --steps 20 --warmup 3
+    run c2_grain_$v "$lib" --mode materialise --cipher grain --steps 4 --warmup 3
+    run c2_mickey_$v "$lib" --mode materialise --cipher mickey2 --steps 3 --warmup 3
   done
 done
