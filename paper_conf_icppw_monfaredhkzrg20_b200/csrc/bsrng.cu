@@ -250,7 +250,7 @@ bsrng_t* bsrng_create_ex(bsrng_cipher cipher, const uint8_t* keys, const uint8_t
     if (cudaMalloc(&h->state, uint64_t(ops->nstate + 1) * h->Gp * 4) != cudaSuccess ||
         cudaMalloc(&h->sliced, sl_words * 4) != cudaSuccess ||
         cudaMalloc(&h->raw, raw_bytes) != cudaSuccess ||
-        cudaMalloc(&h->sched, (1 + h->units + 32) * 4) != cudaSuccess ||
+        cudaMalloc(&h->sched, (1 + h->units + 32 + 1) * 4) != cudaSuccess ||
         (aes && cudaMalloc(&h->rk_dev, 11 * 128 * 4) != cudaSuccess) ||
         cudaMalloc(&h->tail, 32 * 32 * uint64_t(h->key_bytes + h->iv_bytes)) != cudaSuccess) {
         cudaGetLastError();
@@ -489,6 +489,12 @@ void bsrng_destroy(bsrng_t* h)
     if (h->sliced) cudaFree(h->sliced);
     if (h->raw) cudaFree(h->raw);
     if (h->sched) cudaFree(h->sched);
+    if (h->side) {
+        cudaStreamSynchronize(h->side);
+        cudaStreamDestroy(h->side);
+    }
+    if (h->ev_fork) cudaEventDestroy(h->ev_fork);
+    if (h->ev_join) cudaEventDestroy(h->ev_join);
     if (h->bounce) cudaFree(h->bounce);
     if (h->rk_dev) cudaFree(h->rk_dev);
     if (h->tail) cudaFree(h->tail);

@@ -128,7 +128,8 @@ int launch_aes(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st, uint64_t r
 }
 
 // AES ROW_MAJOR with >= 32 blocks per instance: block-lane kernel (aes.cuh).
-int launch_aes_rowmajor_lanes(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st, uint64_t row_stride)
+int launch_aes_rowmajor_lanes(bsrng_t* h, void* out, uint64_t bits, cudaStream_t st, uint64_t row_stride,
+                              uint32_t* ticket)
 {
     auto kern = &bsk::aes_ctr_rowmajor_lanes_kernel;
     bsk::KsArgs a{};
@@ -142,8 +143,8 @@ int launch_aes_rowmajor_lanes(bsrng_t* h, void* out, uint64_t bits, cudaStream_t
     a.row_bytes = row_stride;
     a.units = h->G;  // one warp = 32 instances = one group
     a.persistent = 1;
-    a.ticket = h->sched;
-    a.flags = h->sched + 1;
+    a.ticket = ticket;
+    a.flags = nullptr;  // items are independent
     int occ = h->opt_ctas_per_sm > 0 ? h->opt_ctas_per_sm : 2;
     int occ_max = 1;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_max, kern, 128, 0) != cudaSuccess || occ_max < 1)
@@ -157,7 +158,7 @@ int launch_aes_rowmajor_lanes(bsrng_t* h, void* out, uint64_t bits, cudaStream_t
     const uint64_t seg = ((bits + nseg - 1) / nseg + quantum - 1) / quantum * quantum;
     a.nseg = (bits + seg - 1) / seg;
     a.seg_clocks = seg;
-    cudaError_t e = cudaMemsetAsync(h->sched, 0, sizeof(uint32_t), st);
+    cudaError_t e = cudaMemsetAsync(ticket, 0, sizeof(uint32_t), st);
     if (e != cudaSuccess) return fail(BSRNG_ECUDA, "memset: %s", cudaGetErrorString(e));
     const uint64_t items = a.units * a.nseg;
     const unsigned grid = unsigned(std::min<uint64_t>((items + 3) / 4, uint64_t(h->num_sms) * occ));
@@ -174,11 +175,28 @@ int generate_aes(bsrng_t* h, void* out, uint64_t bits, bsrng_layout layout, cuda
         // ran at 0.44 of the roofline), so it goes to the instance-sliced
         // kernel, writing the rows' last bytes
         const uint64_t main_bits = bits / 4096 * 4096, rem = bits - main_bits;
-        int rc = launch_aes_rowmajor_lanes(h, out, main_bits, st, bits / 8);
-        if (rc == BSRNG_OK && rem)
-            rc = launch_aes<bsk::L_ROW_MAJOR>(h, static_cast<uint8_t*>(out) + main_bits / 8, rem, st, bits / 8,
+        if (!rem) return launch_aes_rowmajor_lanes(h, out, main_bits, st, bits / 8, h->sched);
+        // The remainder (few warp-units, one warp per SMSP, one CTA per SM:
+        // 18% of a paper-shape call run alone) goes first, on the handle's side
+        // stream, so the block-lane kernel's CTAs fill the SMSPs beside it.
+        // The two write disjoint bytes of the rows and only read the state;
+        // each has its own queue ticket.
+        if (!h->side) {
+            if (cudaStreamCreateWithFlags(&h->side, cudaStreamNonBlocking) != cudaSuccess ||
+                cudaEventCreateWithFlags(&h->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
+                cudaEventCreateWithFlags(&h->ev_join, cudaEventDisableTiming) != cudaSuccess)
+                return fail(BSRNG_ECUDA, "side stream / events");
+        }
+        cudaError_t e = cudaEventRecord(h->ev_fork, st);
+        if (e == cudaSuccess) e = cudaStreamWaitEvent(h->side, h->ev_fork, 0);
+        if (e != cudaSuccess) return fail(BSRNG_ECUDA, "fork: %s", cudaGetErrorString(e));
+        int rc = launch_aes<bsk::L_ROW_MAJOR>(h, static_cast<uint8_t*>(out) + main_bits / 8, rem, h->side, bits / 8,
                                               main_bits);
-        return rc;
+        const int rc2 = launch_aes_rowmajor_lanes(h, out, main_bits, st, bits / 8, h->sched + 1 + h->units + 32);
+        e = cudaEventRecord(h->ev_join, h->side);
+        if (e == cudaSuccess) e = cudaStreamWaitEvent(st, h->ev_join, 0);
+        if (e != cudaSuccess) return fail(BSRNG_ECUDA, "join: %s", cudaGetErrorString(e));
+        return rc != BSRNG_OK ? rc : rc2;
     }
     switch (layout) {
     case BSRNG_ROW_MAJOR: return launch_aes<bsk::L_ROW_MAJOR>(h, out, bits, st);

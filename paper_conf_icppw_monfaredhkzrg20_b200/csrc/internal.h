@@ -62,7 +62,11 @@ struct bsrng {
     uint32_t* sliced = nullptr;  // key [KB][Gp] then iv [IVB][Gp] (unfused init only)
     uint8_t* raw = nullptr;      // keys [Gp*32][key_bytes] then ivs at raw + iv_off (zero-padded)
     uint64_t iv_off = 0;         // per-instance regions padded to Gp*32 rows (zeroed), 16 B aligned
-    uint32_t* sched = nullptr;   // [1 + units]: ticket, flags; then [32] scratch
+    uint32_t* sched = nullptr;   // [1 + units]: ticket, flags; then [32] scratch; then [1] second ticket
+    // AES ROW_MAJOR: the instance-sliced remainder kernel runs on this side
+    // stream beside the block-lane kernel (fork / join events on the caller's stream)
+    cudaStream_t side = nullptr;
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     uint8_t* bounce = nullptr;   // generate_host staging
     uint64_t bounce_bytes = 0;
     // host inputs are copied into this handle-owned pinned buffer before the

@@ -1,8 +1,8 @@
 #!/bin/bash
-# TMEM addresses as warp-uniform values (one UR per transpose, no R2UR per STTM).  Parity, A/B vs HEAD.
+# AES ROW_MAJOR: remainder kernel on a side stream beside the block-lane kernel.  Parity, A/B.
 set -u
-D=gpurun_out/g26; mkdir -p $D
-timeout 900 python -m pytest tests/test_gpu_api.py tests/test_gpu_random.py tests/test_gpu_rowmajor_items.py tests/test_gpu_bounds.py -m gpu -q -p no:cacheprovider > $D/pytest.txt 2>&1
+D=gpurun_out/g28; mkdir -p $D
+timeout 900 python -m pytest tests/test_gpu_aes.py tests/test_gpu_contract.py tests/test_gpu_bounds.py tests/test_gpu_rowmajor_items.py tests/test_gpu_api.py tests/test_gpu_random.py -m gpu -q -p no:cacheprovider > $D/pytest.txt 2>&1
 echo "pytest exit $?" >> $D/pytest.txt
 run() {  # name lib args...
   local name=$1 lib=$2; shift 2
@@ -12,10 +12,7 @@ run() {  # name lib args...
 for rep in 1 2; do
   for v in new old; do
     lib=""; [ $v = old ] && lib=tools/experiments/ab/old.so
-    run c4_grain_$v "$lib" --mode materialise --cipher grain --workload c4 --steps 1000 --warmup 20
-    run c4_mickey_$v "$lib" --mode materialise --cipher mickey2 --workload c4 --steps 300 --warmup 10
-    run lfsr_$v "$lib" --mode materialise --cipher lfsr128 --steps 20 --warmup 3
-    run c2_grain_$v "$lib" --mode materialise --cipher grain --steps 4 --warmup 3
-    run c2_mickey_$v "$lib" --mode materialise --cipher mickey2 --steps 3 --warmup 3
+    run c4_aes_$v "$lib" --mode materialise --cipher aes128ctr --workload c4 --steps 2000 --warmup 20
   done
 done
+run c2_aes_new "" --mode materialise --cipher aes128ctr --steps 10 --warmup 3
