@@ -146,7 +146,12 @@ int bsrng_rekey(bsrng_t* h, const uint8_t* keys, const uint8_t* ivs, uint32_t fl
  *          more than 2^31 bits per instance run as several time segments of
  *          one launch (the same result as one pass).
  *   stream: must belong to the handle's device (else EINVAL); NULL = the
- *          legacy default stream.
+ *          legacy default stream.  AES ROW_MAJOR calls of >= 4096 bits with a
+ *          < 4096-bit remainder run that remainder on a handle-owned side
+ *          stream forked from and joined back into `stream` by events, so
+ *          the call stays ordered after earlier and before later work on
+ *          `stream` (and is capturable in a CUDA graph).  Calls on one handle
+ *          must not run concurrently on different streams.
  * Errors: EINVAL (NULL, alignment, bits, layout, stream), ERANGE (cumulative
  * bits per instance above the cipher's limit, see BSRNG_ERANGE), ECUDA.
  */
