@@ -24,6 +24,11 @@
 //     other writer's flush of the same lines follows within a few blocks, so
 //     L2 (evict_last) sees whole 128 B lines.
 //
+// A writer takes its blocks in pairs (one full-barrier wait per pair) and
+// transposes two consecutive blocks of one item together (F_PAIR), writing
+// each row's two words with one tcgen05.st.32x32b.x2: twice the independent
+// work for a latency-bound lone warp (LFSR C2 27.3 -> 28.7 Tb/s).
+//
 // Ring sequence: block seq sits in ring slot seq % 16 and belongs to writer
 // (seq >> 3) & 1, so each writer walks its own 8 slots; the clock-loop warp
 // keeps seq = B (mod 16) by publishing skip blocks at item starts, which
